@@ -1,0 +1,210 @@
+/*
+ * ctxb.h -- C ABI of the B200-native CTXBack context save / restore path.
+ *
+ * CTXBack (Ji & Wang, IPDPS 2021; `P:n` = line n of reference PAPER.md) lets a
+ * preempted warp save the register context of a *preceding* instruction (its
+ * flashback-point) instead of the current one, and on resume reload that
+ * context, revert and re-execute the in-between instructions.
+ *
+ * This library implements, for kernels written in the small register IR of
+ * DESIGN.md ("IR v1"):
+ *   - the compile-time pass: liveness, flashback-point search with
+ *     the relaxed condition, instruction reverting and on-chip scalar backup,
+ *     per-site plan selection, and generation of one dedicated preemption
+ *     routine and one dedicated resume routine per poll site, as sm_100a CUDA
+ *     compiled with NVRTC                                 -> ctxb_analyze
+ *   - the runtime: launching the generated kernel, raising the
+ *     preemption signal, draining the warps into a caller-owned context
+ *     buffer, and resuming them                          -> ctxb_launch /
+ *                                                           ctxb_preempt /
+ *                                                           ctxb_resume
+ *
+ * Conventions
+ *   - Every function returns an int status: CTXB_OK (0) or a negative
+ *     CTXB_E_* code.  No C++ exception crosses the ABI.  ctxb_last_error()
+ *     returns a thread-local message describing the last failure.
+ *   - Handles (ctxb_program, ctxb_run) are created and destroyed by the
+ *     library.  Device buffers and the context buffer are owned by the
+ *     caller (e.g. torch tensors, passed as raw device pointers); they must
+ *     outlive every run that uses them.
+ *   - Streams are borrowed: `stream` arguments are CUstream / cudaStream_t
+ *     handles of the current device's primary context passed as void*
+ *     (NULL = legacy default stream).  No torch type appears here.
+ *   - There is no CPU fallback: ctxb_launch and friends fail with
+ *     CTXB_E_CUDA when no CUDA device / driver is present.  ctxb_analyze needs
+ *     only NVRTC (it compiles without a GPU) unless CTXB_DEBUG_NO_COMPILE.
+ */
+#ifndef CTXB_H
+#define CTXB_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- status codes ------------------------------------------------------ */
+#define CTXB_OK                  0
+#define CTXB_E_INVALID_ARG      -1   /* NULL handle / out pointer, bad index, bad size   */
+#define CTXB_E_PARSE            -2   /* IR text does not follow DESIGN.md "IR v1"        */
+#define CTXB_E_ANALYSIS         -3   /* internal analysis failure (a bug)                */
+#define CTXB_E_NVRTC            -4   /* NVRTC missing or generated CUDA failed to build  */
+#define CTXB_E_CUDA             -5   /* driver missing or a CUDA driver call failed      */
+#define CTXB_E_STATE            -6   /* preempt on a finished run, resume on a run that
+                                        is not preempted, ...                            */
+#define CTXB_E_BUFFER_TOO_SMALL -7   /* context buffer / output buffer too small         */
+
+/* ---- options (P:34-36 three techniques; P:337 compared schemes) ---------- */
+#define CTXB_RELAXED  1u  /* relaxed flashback-point condition, Alg. 1 */
+#define CTXB_REVERT   2u  /* instruction reverting, Alg. 2            */
+#define CTXB_OSRB     4u  /* on-chip scalar register backup           */
+#define CTXB_ALL      7u
+
+#define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
+#define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */
+#define CTXB_MODE_FULL    2u /* save every declared IR register (FULL_IR)        */
+#define CTXB_MODE_FULL_HW 3u /* FULL_IR padded to the compiled kernel's register
+                                count per thread: the analogue of the BASELINE
+                                routine that swaps all occupied registers */
+
+#define CTXB_POLL_EVERY_INSTR 0u /* a poll site before every IR instruction   */
+#define CTXB_POLL_EVERY_N     1u /* before BB-local index i, i % N == 0, i > 0,
+                                    and before every backward branch          */
+#define CTXB_POLL_EXPLICIT    2u /* before the IR's `poll` markers             */
+
+#define CTXB_DEBUG_FORCED     1u /* poll sites compare the warp's poll-visit count
+                                    with a per-warp target instead of reading the
+                                    preemption flag (deterministic tests)      */
+#define CTXB_DEBUG_POISON     2u /* the resume kernel fills every IR register with
+                                    a poison pattern before restoring          */
+#define CTXB_DEBUG_NO_POLLS   4u /* compile poll sites out (overhead baseline;
+                                    the kernel cannot be preempted)            */
+#define CTXB_DEBUG_NO_COMPILE 8u /* analysis + code generation only            */
+
+typedef struct {
+  uint32_t flags;       /* CTXB_RELAXED | CTXB_REVERT | CTXB_OSRB                */
+  uint32_t mode;        /* CTXB_MODE_*                                           */
+  uint32_t poll_policy; /* CTXB_POLL_*                                           */
+  uint32_t poll_every;  /* N for CTXB_POLL_EVERY_N                               */
+  uint32_t debug;       /* CTXB_DEBUG_* bits                                     */
+} ctxb_options;
+
+typedef struct ctxb_program ctxb_program; /* analysed IR kernel + module; library-owned */
+typedef struct ctxb_run ctxb_run;         /* one launch and its preempt/resume history   */
+
+/* Per poll-site plan summary (one dedicated routine pair per site). */
+typedef struct {
+  uint32_t c;               /* site = before IR instruction c (R-1)           */
+  uint32_t p;               /* chosen flashback-point instruction (p <= c)          */
+  uint32_t n_vec;           /* saved vector values (128 B per warp each, R-8)       */
+  uint32_t n_scalar;        /* saved scalar values (4 B per warp each)              */
+  uint32_t n_revert_pre;    /* reverting instructions run at preempt (Alg. 2)       */
+  uint32_t n_revert_res;    /* reverting instructions run at resume                 */
+  uint32_t n_reexec;        /* re-executed instructions at resume (Alg. 1)          */
+  uint32_t payload_bytes_per_warp; /* 128*n_vec + 4*n_scalar                        */
+  uint32_t live_bytes_per_warp;    /* the LIVE plan of the same site (fallback)     */
+} ctxb_site_info_t;
+
+typedef struct {
+  uint32_t n_instrs, nv, ns, block, n_buffers, n_uniforms, n_sites, n_backups;
+  uint32_t max_payload_bytes_per_warp; /* over every plan incl. LIVE fallbacks       */
+  uint32_t full_ir_bytes_per_warp;     /* 128*nv + 4*ns                              */
+  uint32_t num_regs;                   /* ptxas registers/thread (0 if not compiled) */
+  uint32_t compiled;                   /* 1 if a cubin was produced                  */
+  double analyze_ms, codegen_ms, compile_ms;
+} ctxb_program_info_t;
+
+typedef struct {
+  double latency_us;         /* device: max t_saved - min t_flag_seen over preempted
+                                warps (%globaltimer), "elapsed time before
+                                releasing the GPU"                                 */
+  double host_us;            /* host: flag write issued -> victim stream drained   */
+  uint32_t warps_preempted, warps_done, blocks_preempted;
+  uint64_t payload_bytes;    /* sum of saved payload over preempted warps          */
+  uint64_t header_bytes;     /* 16 B per preempted warp                             */
+} ctxb_preempt_stats;
+
+typedef struct {
+  double resume_us;          /* device: max t_site_reached - min t_resume_entry    */
+  uint32_t warps_resumed;
+} ctxb_resume_stats;
+
+const char* ctxb_last_error(void);
+const char* ctxb_version(void);
+
+/* Parse + analyse + generate + compile.  `ir_text` need not be
+ * NUL-terminated (`len` bytes are read).  opts == NULL means
+ * {CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0}.
+ * Errors: _INVALID_ARG, _PARSE, _ANALYSIS, _NVRTC. */
+int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb_program** out);
+int ctxb_program_destroy(ctxb_program* prog);
+int ctxb_program_info(const ctxb_program* prog, ctxb_program_info_t* out);
+int ctxb_num_sites(const ctxb_program* prog, uint32_t* n);
+int ctxb_site_info(const ctxb_program* prog, uint32_t site, ctxb_site_info_t* out);
+/* OSRB-selected scalar defs (instruction indices), up to `cap`; *n = total. */
+int ctxb_backups(const ctxb_program* prog, uint32_t* idx, uint32_t cap, uint32_t* n);
+/* Canonical text of a site's plan, NUL-terminated;
+ * *len = required size incl. NUL; _BUFFER_TOO_SMALL if cap < *len. */
+int ctxb_site_plan_text(const ctxb_program* prog, uint32_t site, int live, char* buf, size_t cap,
+                        size_t* len);
+/* The generated CUDA C++ source (same buffer convention). */
+int ctxb_generated_source(const ctxb_program* prog, char* buf, size_t cap, size_t* len);
+
+/* Bytes of device memory a context buffer for `grid_blocks` blocks needs:
+ * 16 B header per warp + per-warp payload slots. */
+int ctxb_context_capacity(const ctxb_program* prog, uint32_t grid_blocks, uint64_t* bytes);
+
+/* Launch the generated kernel ("if no preemption occurs, CTXBack incurs
+ * no extra work except OSRB").  buffers[i] = device pointer of the i-th
+ * `.buffer` in IR order (u32 elements); uniforms[i] = value of the i-th
+ * `.uniform`.  ctx_buf: caller-owned device memory of >= capacity bytes.
+ * forced_targets (CTXB_DEBUG_FORCED programs only, else NULL): host array of
+ * grid_blocks*block/32 u32, the 0-based poll visit at which each warp is
+ * preempted (0xFFFFFFFF = never).  The launch is asynchronous on `stream`. */
+int ctxb_launch(ctxb_program* prog, uint32_t grid_blocks, void* const* buffers,
+                const uint32_t* uniforms, void* ctx_buf, uint64_t ctx_buf_bytes, void* stream,
+                const uint32_t* forced_targets, ctxb_run** out);
+
+/* Raise the preemption signal (a device flag written by `ctrl_stream`, which
+ * must not be the run's stream), wait until every warp of the run has either
+ * saved its context and exited or finished, clear the flag.  Fills
+ * `stats` if non-NULL.  _STATE if the run is not running. */
+int ctxb_preempt(ctxb_run* run, void* ctrl_stream, ctxb_preempt_stats* stats);
+
+/* Relaunch the same grid as a resume kernel: each preempted warp reloads its
+ * context, reverts / re-executes to its site and continues; finished warps
+ * exit at once.  forced_targets as in ctxb_launch.  Asynchronous.
+ * _STATE unless the run is preempted. */
+int ctxb_resume(ctxb_run* run, void* stream, const uint32_t* forced_targets);
+
+/* Wait for the run's current launch; *finished = 1 if every warp is done,
+ * 0 if some warps were preempted (forced mode or a racing ctxb_preempt). */
+int ctxb_wait(ctxb_run* run, int* finished);
+
+/* Device timings of the last resume launch (valid after ctxb_wait/preempt). */
+int ctxb_resume_stats_get(const ctxb_run* run, ctxb_resume_stats* out);
+
+/* Sum over warps of the last preemption: payload bytes, header bytes and the
+ * number of thread blocks with >= 1 preempted warp (P:343 context size). */
+int ctxb_context_bytes(const ctxb_run* run, uint64_t* payload, uint64_t* header,
+                       uint32_t* n_tb_preempted);
+
+/* Copy the per-warp headers {site | live<<31, payload_bytes, state, epoch}
+ * (4 u32 per warp) of the last completed launch into host memory. */
+int ctxb_read_headers(const ctxb_run* run, uint32_t* host_out, uint64_t n_words);
+/* Copy the per-warp %globaltimer stamps {t_flag_seen, t_saved, t_resume_entry,
+ * t_site_reached} (4 u64 per warp). */
+int ctxb_read_stamps(const ctxb_run* run, uint64_t* host_out, uint64_t n_words);
+
+int ctxb_run_destroy(ctxb_run* run);
+
+/* Header `state` values. */
+#define CTXB_STATE_NONE      0u
+#define CTXB_STATE_PREEMPTED 1u
+#define CTXB_STATE_DONE      2u
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CTXB_H */

@@ -356,7 +356,7 @@ class Machine:
         nbytes = sum(128 if v[0][0] == "v" else 4 for v in ctx)
         assert nbytes == plan.payload_bytes
         self.records.append(dict(warp=int(self.warp_ids[w]), site=c, kind=plan.kind,
-                                 bytes=plan.payload_bytes, p=plan.p))
+                                 bytes=plan.payload_bytes, p=plan.p, launch=self.cur_launch))
         # poison every register and slot of the warp (nothing but ctx survives)
         self.V[:, w, :] = self.rng.integers(0, 1 << 32, size=self.V[:, w, :].shape, dtype=np.uint32)
         self.S[:, w] = self.rng.integers(0, 1 << 32, size=self.S[:, w].shape, dtype=np.uint32)
@@ -523,6 +523,7 @@ class Machine:
         not preempted.  Returns the final buffers."""
         launch = 0
         while True:
+            self.cur_launch = launch
             t = np.full(self.nW, NEVER, dtype=np.int64)
             if launch < len(schedule) and schedule[launch] is not None:
                 s = np.asarray(schedule[launch], dtype=np.int64)

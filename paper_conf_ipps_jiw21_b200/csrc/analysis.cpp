@@ -1,0 +1,650 @@
+// Compile-time flashback analysis in the normative reading CTXB-R1
+// (SURVEY §8(c2)).  Paper passages:
+//   liveness = register context of an instruction .................. P:80
+//   window [I_prec, I_cur), signal handled before I_cur ............. P:74 (R-1)
+//   relaxed condition, Alg. 1 ....................................... P:88-152 (R-2)
+//   instruction reverting, Alg. 2 ................................... P:154-231 (R-5, R-6)
+//   on-chip scalar register backup .................................. P:257-269 (R-7)
+//   combined fixpoint ............................................... P:271-303 (R-9)
+//   windows inside the basic block and idempotent region ............ P:305 (R-3)
+//   least-latency flashback-point per instruction ................... P:313, P:337 (R-10)
+//   context incl. results restored by saving/reloading .............. P:343 (R-8)
+#include <algorithm>
+#include <functional>
+#include <set>
+#include <sstream>
+
+#include "ctxb_internal.h"
+
+namespace ctxb {
+namespace {
+
+constexpr uint32_t F_RELAXED = 1, F_REVERT = 2, F_OSRB = 4;
+constexpr uint32_t VEC_B = 128, SCA_B = 4;
+
+bool is_alu(Op o) {
+  switch (o) {
+    case Op::Mov: case Op::Not: case Op::Neg: case Op::I2F: case Op::U2F: case Op::F2I:
+    case Op::IAdd: case Op::ISub: case Op::IMul: case Op::And: case Op::Or: case Op::Xor:
+    case Op::Shl: case Op::Shr: case Op::Sar: case Op::RotL: case Op::RotR: case Op::UMin:
+    case Op::UMax: case Op::IMin: case Op::IMax: case Op::FAdd: case Op::FSub: case Op::FMul:
+    case Op::FFma: case Op::IMad: case Op::Sel: case Op::Setp:
+      return true;
+    default:
+      return false;
+  }
+}
+
+// R-4: ALU ops and loads from read-only buffers can be re-executed.
+bool reexec_op(const Program& P, const Instr& I) {
+  if (is_alu(I.op)) return true;
+  if (I.op == Op::Ldg) return P.buf_kinds[I.buf] == B_RO;
+  return false;
+}
+
+int regid(const Program& P, const Operand& o) { return o.kind == OK::V ? (int)o.val : P.nv + (int)o.val; }
+
+// R-5: r' = op(r, {R}) with a bit-exact inverse.  Fills kind and the
+// non-shared operands (in operand order).
+bool revert_spec(const Program& P, const Instr& I, int r, RevKind* kind, std::vector<Operand>* others) {
+  if (I.defreg != r || I.dst.kind == OK::None) return false;
+  if (I.guard.kind != OK::None || I.idx.kind != OK::None) return false;
+  int cnt = 0;
+  for (auto& o : I.srcs)
+    if (o.is_reg() && regid(P, o) == r) cnt++;
+  if (cnt != 1) return false;
+  others->clear();
+  if (I.op == Op::Not || I.op == Op::Neg) {
+    *kind = I.op == Op::Not ? RV_NOT_D : RV_NEG_D;
+    return true;
+  }
+  if (I.srcs.size() != 2) return false;
+  const Operand& a = I.srcs[0];
+  const Operand& b = I.srcs[1];
+  bool a_is = a.is_reg() && regid(P, a) == r;
+  const Operand& other = a_is ? b : a;
+  switch (I.op) {
+    case Op::IAdd: *kind = RV_SUB_D; others->push_back(other); return true;
+    case Op::ISub:
+      *kind = a_is ? RV_ADD_D : RV_RSUB_D;
+      others->push_back(other);
+      return true;
+    case Op::Xor: *kind = RV_XOR_D; others->push_back(other); return true;
+    case Op::IMul:
+      if (other.kind == OK::Imm && (other.val & 1u)) {
+        *kind = RV_MULINV;
+        others->push_back(other);
+        return true;
+      }
+      return false;
+    case Op::RotL: case Op::RotR:
+      if (a_is && b.kind == OK::Imm) {
+        *kind = I.op == Op::RotL ? RV_ROTR : RV_ROTL;
+        others->push_back(b);
+        return true;
+      }
+      return false;
+    default:
+      return false;
+  }
+}
+
+struct Liveness {
+  std::vector<std::vector<uint8_t>> in, out;
+};
+
+Liveness liveness(const Program& P) {
+  int R = P.nregs(), nb = (int)P.bbs.size();
+  std::vector<std::vector<uint8_t>> use(nb, std::vector<uint8_t>(R, 0)), def(nb, std::vector<uint8_t>(R, 0)),
+      lin(nb, std::vector<uint8_t>(R, 0)), lout(nb, std::vector<uint8_t>(R, 0));
+  for (int b = 0; b < nb; b++)
+    for (int i = P.bbs[b].first; i < P.bbs[b].second; i++) {
+      for (int u : P.ins[i].uses)
+        if (!def[b][u]) use[b][u] = 1;
+      if (P.ins[i].defreg >= 0) def[b][P.ins[i].defreg] = 1;
+    }
+  bool changed = true;
+  while (changed) {
+    changed = false;
+    for (int b = nb - 1; b >= 0; b--) {
+      std::vector<uint8_t> o(R, 0), i_(R, 0);
+      for (int s : P.succ[b])
+        for (int r = 0; r < R; r++) o[r] |= lin[s][r];
+      for (int r = 0; r < R; r++) i_[r] = use[b][r] | (o[r] & !def[b][r]);
+      if (o != lout[b] || i_ != lin[b]) {
+        lout[b] = o;
+        lin[b] = i_;
+        changed = true;
+      }
+    }
+  }
+  Liveness L;
+  int n = (int)P.ins.size();
+  L.in.assign(n, {});
+  L.out.assign(n, {});
+  for (int b = 0; b < nb; b++) {
+    std::vector<uint8_t> cur = lout[b];
+    for (int i = P.bbs[b].second - 1; i >= P.bbs[b].first; i--) {
+      L.out[i] = cur;
+      if (P.ins[i].defreg >= 0) cur[P.ins[i].defreg] = 0;
+      for (int u : P.ins[i].uses) cur[u] = 1;
+      L.in[i] = cur;
+    }
+  }
+  return L;
+}
+
+// h(c): max(BB start, idempotent-region start); a region starts after every
+// atomic and at a store to a buffer loaded earlier in the region (R-3).
+std::vector<int> region_heads(const Program& P) {
+  std::vector<int> heads(P.ins.size(), 0);
+  for (auto [s, e] : P.bbs) {
+    int head = s;
+    std::set<int> loaded;
+    for (int c = s; c < e; c++) {
+      heads[c] = head;
+      const Instr& I = P.ins[c];
+      if (I.op == Op::AtomAdd || I.op == Op::AtomCas) {
+        head = c + 1;
+        loaded.clear();
+      } else if (I.op == Op::Stg && loaded.count(I.buf)) {
+        head = c;
+        loaded.clear();
+      } else if (I.op == Op::Ldg) {
+        loaded.insert(I.buf);
+      }
+    }
+  }
+  return heads;
+}
+
+std::vector<int> sites_for(const Program& P, const Options& opt) {
+  std::vector<int> out;
+  if (opt.policy == 0) {
+    for (int i = 0; i < (int)P.ins.size(); i++) out.push_back(i);
+  } else if (opt.policy == 2) {
+    std::set<int> s(P.explicit_sites.begin(), P.explicit_sites.end());
+    out.assign(s.begin(), s.end());
+  } else {
+    int N = (int)std::max<uint32_t>(1, opt.every);
+    std::set<int> s;
+    for (int b = 0; b < (int)P.bbs.size(); b++) {
+      auto [s0, e0] = P.bbs[b];
+      for (int i = s0 + N; i < e0; i += N) s.insert(i);
+      const Instr& last = P.ins[e0 - 1];
+      if ((last.op == Op::Bra || last.op == Op::Brnz || last.op == Op::Brz) && last.target_bb <= b) s.insert(e0 - 1);
+    }
+    out.assign(s.begin(), s.end());
+  }
+  return out;
+}
+
+struct Deriv {
+  SK k = SK::C;
+  int arg = -1;
+  bool present = false;
+};
+
+// Per-BB sorted definition positions of every register.
+struct DefIndex {
+  std::vector<std::vector<std::vector<int>>> pos;  // [bb][reg] -> positions
+  explicit DefIndex(const Program& P) {
+    pos.assign(P.bbs.size(), std::vector<std::vector<int>>(P.nregs()));
+    for (int i = 0; i < (int)P.ins.size(); i++)
+      if (P.ins[i].defreg >= 0) pos[P.bb_of[i]][P.ins[i].defreg].push_back(i);
+  }
+};
+
+// One (site c, flashback-point p) evaluation of the CTXB-R1 sweep.
+class Window {
+ public:
+  Window(const Program& P, const Liveness& L, const DefIndex& D, int p, int c, const std::vector<int>& backups,
+         uint32_t flags)
+      : P(P), L(L), D(D), p(p), c(c), flags(flags) {
+    bb = P.bb_of[std::min(c, (int)P.ins.size() - 1)];
+    if (c > p) bb = P.bb_of[p];
+    int R = P.nregs();
+    vpre.assign(R, {});
+    vdef.assign(c - p, {});
+    reexec.assign(c - p, 0);
+    for (int r = 0; r < R; r++) set_valid({r, rd(r, c)}, {SK::C, -1, true});
+    std::vector<int> bs(backups);
+    std::sort(bs.begin(), bs.end());
+    for (int m : bs)
+      if (p <= m && m < c) {
+        int s = P.ins[m].defreg;
+        Val v{s, rd(s, m)};
+        if (!valid(v)) set_valid(v, {SK::B, m, true});
+      }
+  }
+
+  int rd(int r, int t) const {  // last def of r in [p, t), else PRE
+    if (t <= p) return PRE;
+    const auto& v = D.pos[P.bb_of[p < (int)P.ins.size() ? p : t - 1]][r];
+    auto it = std::lower_bound(v.begin(), v.end(), t);
+    if (it == v.begin()) return PRE;
+    --it;
+    return *it >= p ? *it : PRE;
+  }
+  int nd(int r, int t) const {  // first def of r in [t, c), else -1
+    if (t >= c) return -1;
+    const auto& v = D.pos[P.bb_of[t]][r];
+    auto it = std::lower_bound(v.begin(), v.end(), t);
+    if (it == v.end() || *it >= c) return -1;
+    return *it;
+  }
+  bool is_current(const Val& v) const { return nd(v.r, v.d == PRE ? p : v.d + 1) < 0; }
+  bool valid(const Val& v) const { return v.d == PRE ? vpre[v.r].present : vdef[v.d - p].present; }
+  const Deriv& deriv(const Val& v) const { return v.d == PRE ? vpre[v.r] : vdef[v.d - p]; }
+  void set_valid(const Val& v, Deriv d) {
+    d.present = true;
+    if (v.d == PRE)
+      vpre[v.r] = d;
+    else
+      vdef[v.d - p] = d;
+  }
+  std::vector<Val> opvals(int j) const {
+    std::vector<Val> out;
+    for (int u : P.ins[j].uses) out.push_back({u, rd(u, j)});
+    return out;
+  }
+  bool liveout_def(int j) const {
+    int r = P.ins[j].defreg;
+    return r >= 0 && L.out[j][r];
+  }
+  bool reexec_kind(int j) const { return liveout_def(j) && reexec_op(P, P.ins[j]); }
+  Supply to_supply(const Deriv& d) const { return {d.k, d.arg}; }
+  Supply supply_of(const Val& v) const {
+    if (v.d != PRE && reexec[v.d - p]) return {SK::X, v.d};
+    return to_supply(deriv(v));
+  }
+
+  bool try_revert(const Val& v) {
+    if (!(flags & F_REVERT)) return false;
+    int m = nd(v.r, v.d == PRE ? p : v.d + 1);
+    if (m < 0) return false;
+    RevertRec rec;
+    if (!revert_spec(P, P.ins[m], v.r, &rec.kind, &rec.others)) return false;
+    rec.v = v;
+    rec.m = m;
+    rec.inputs.push_back({v.r, m});
+    for (auto& o : rec.others)
+      if (o.is_reg()) {
+        int u = regid(P, o);
+        rec.inputs.push_back({u, rd(u, m)});
+      }
+    for (auto& x : rec.inputs) {
+      if (is_current(x)) {
+        rec.supplies.push_back({SK::C, -1});
+      } else if (valid(x)) {
+        rec.supplies.push_back(supply_of(x));
+      } else if (try_revert(x)) {
+        rec.supplies.push_back(to_supply(deriv(x)));
+      } else {
+        return false;
+      }
+    }
+    set_valid(v, {SK::R, m, true});
+    revs[v] = rec;
+    events.push_back({false, m, v});
+    return true;
+  }
+
+  void sweep() {
+    bool changed = true;
+    while (changed) {
+      changed = false;
+      for (int j = p; j < c; j++) {
+        if (reexec[j - p] || !reexec_kind(j)) continue;
+        auto ov = opvals(j);
+        for (auto& x : ov)
+          if (!valid(x) && try_revert(x)) changed = true;
+        bool all = true;
+        for (auto& x : ov) all = all && valid(x);
+        if (all) {
+          std::vector<Supply> sup;
+          for (auto& x : ov) sup.push_back(supply_of(x));
+          reexec[j - p] = 1;
+          rx_supply[j] = sup;
+          events.push_back({true, j, {P.ins[j].defreg, j}});
+          Val v{P.ins[j].defreg, j};
+          if (!valid(v)) set_valid(v, {SK::X, j, true});
+          changed = true;
+        }
+      }
+      for (int j = p; j < c; j++)
+        if (liveout_def(j)) {
+          Val v{P.ins[j].defreg, j};
+          if (!valid(v) && try_revert(v)) changed = true;
+        }
+    }
+  }
+
+  bool feasible() const {
+    for (int j = p; j < c; j++)
+      if (liveout_def(j) && !valid({P.ins[j].defreg, j})) return false;
+    return true;
+  }
+
+  std::vector<std::pair<Val, Supply>> demands() const {
+    std::vector<std::pair<Val, Supply>> out;
+    for (int j = p; j < c; j++)
+      if (reexec[j - p]) {
+        auto ov = opvals(j);
+        const auto& sup = rx_supply.at(j);
+        for (size_t k = 0; k < ov.size(); k++) out.push_back({ov[k], sup[k]});
+      }
+    for (int j = p; j < c; j++)
+      if (liveout_def(j) && !reexec[j - p]) {
+        Val v{P.ins[j].defreg, j};
+        out.push_back({v, to_supply(deriv(v))});
+      }
+    for (int r = 0; r < P.nregs(); r++)
+      if (L.in[c][r] && rd(r, c) == PRE) out.push_back({{r, PRE}, {SK::C, -1}});
+    return out;
+  }
+
+  struct SRes {
+    std::map<Val, char> S;
+    std::set<Val> used_res, used_pre;
+  };
+
+  SRes compute_S(const std::map<Val, char>& pos) const {
+    SRes R;
+    std::function<void(const Val&)> pre_closure = [&](const Val& v) {
+      if (R.used_pre.count(v)) return;
+      R.used_pre.insert(v);
+      const RevertRec& rec = revs.at(v);
+      for (size_t k = 0; k < rec.inputs.size(); k++)
+        if (rec.supplies[k].k == SK::R) pre_closure(rec.inputs[k]);
+    };
+    std::function<void(const Val&, const Supply&)> demand = [&](const Val& v, const Supply& s) {
+      switch (s.k) {
+        case SK::C: R.S.emplace(v, 'C'); break;
+        case SK::B: R.S.emplace(v, 'B'); break;
+        case SK::X: break;
+        case SK::R: {
+          auto it = pos.find(v);
+          char ps = it == pos.end() ? 'R' : it->second;
+          if (ps == 'P') {
+            R.S.emplace(v, 'P');
+            pre_closure(v);
+          } else {
+            if (R.used_res.count(v)) return;
+            R.used_res.insert(v);
+            const RevertRec& rec = revs.at(v);
+            for (size_t k = 0; k < rec.inputs.size(); k++) demand(rec.inputs[k], rec.supplies[k]);
+          }
+          break;
+        }
+      }
+    };
+    for (auto& [v, s] : demands()) demand(v, s);
+    return R;
+  }
+
+  uint32_t bytes_of(const std::map<Val, char>& S) const {
+    uint32_t b = 0;
+    for (auto& [v, src] : S) b += P.is_vec(v.r) ? VEC_B : SCA_B;
+    return b;
+  }
+
+  Plan plan(int kind) const {
+    std::map<Val, char> pos;
+    for (auto& [v, rec] : revs) pos[v] = 'R';
+    SRes r0 = compute_S(pos);
+    std::vector<Val> order(r0.used_res.begin(), r0.used_res.end());
+    std::stable_sort(order.begin(), order.end(),
+                     [&](const Val& a, const Val& b) { return revs.at(a).m > revs.at(b).m; });
+    for (const Val& v : order) {
+      const RevertRec& rec = revs.at(v);
+      bool forced = false;
+      for (size_t k = 0; k < rec.inputs.size(); k++) {
+        const Supply& s = rec.supplies[k];
+        if (s.k == SK::X || (s.k == SK::R && pos.at(rec.inputs[k]) == 'R')) forced = true;
+      }
+      if (forced) continue;
+      pos[v] = 'P';
+      uint32_t bP = bytes_of(compute_S(pos).S);
+      pos[v] = 'R';
+      uint32_t bR = bytes_of(compute_S(pos).S);
+      if (bP < bR) pos[v] = 'P';
+    }
+    SRes fin = compute_S(pos);
+    Plan pl;
+    pl.valid = true;
+    pl.c = c;
+    pl.p = p;
+    pl.kind = kind;
+    for (auto& [v, src] : fin.S) {
+      SavedVal sv{src, v, -1};
+      if (src == 'B') sv.bkp_m = deriv(v).arg;
+      pl.saved.push_back(sv);
+    }
+    std::sort(pl.saved.begin(), pl.saved.end(), [](const SavedVal& a, const SavedVal& b) {
+      if (a.v.r != b.v.r) return a.v.r < b.v.r;
+      if (a.v.d != b.v.d) return a.v.d < b.v.d;
+      return a.src < b.src;
+    });
+    std::vector<Val> pre(fin.used_pre.begin(), fin.used_pre.end());
+    std::stable_sort(pre.begin(), pre.end(), [&](const Val& a, const Val& b) { return revs.at(a).m > revs.at(b).m; });
+    for (auto& v : pre) pl.pre_reverts.push_back(revs.at(v));
+    for (auto& e : events)
+      if (e.is_x || fin.used_res.count(e.v)) pl.schedule.push_back(e);
+    pl.reexec_supply = rx_supply;
+    pl.revert_info = revs;
+    for (int r = 0; r < P.nregs(); r++)
+      if (L.in[c][r]) {
+        int d = rd(r, c);
+        pl.final_.push_back({r, d == PRE ? Supply{SK::C, -1} : supply_of({r, d})});
+      }
+    pl.payload_bytes = bytes_of(fin.S);
+    for (auto& [v, src] : fin.S) (P.is_vec(v.r) ? pl.n_vec : pl.n_sca)++;
+    pl.n_rev_pre = (uint32_t)fin.used_pre.size();
+    pl.n_rev_res = (uint32_t)fin.used_res.size();
+    uint32_t nx = 0;
+    for (auto x : reexec) nx += x;
+    pl.n_reexec = nx;
+    return pl;
+  }
+
+  const Program& P;
+  const Liveness& L;
+  const DefIndex& D;
+  int p, c, bb;
+  uint32_t flags;
+  std::vector<Deriv> vpre, vdef;
+  std::vector<uint8_t> reexec;
+  std::map<int, std::vector<Supply>> rx_supply;
+  std::map<Val, RevertRec> revs;
+  std::vector<Event> events;
+};
+
+// Basic condition: R_prec not overwritten in [I_prec, I_cur) and
+// every result-producing instruction re-executable; S = LIVE_IN(p).
+Plan basic_plan(const Program& P, const Liveness& L, const DefIndex& D, int p, int c) {
+  for (int j = p; j < c; j++) {
+    int r = P.ins[j].defreg;
+    if (r < 0) continue;
+    if (L.in[p][r] || !reexec_op(P, P.ins[j])) return Plan{};
+  }
+  Window w(P, L, D, p, c, {}, 0);
+  for (int j = p; j < c; j++)
+    if (P.ins[j].defreg >= 0) {
+      std::vector<Supply> sup;
+      for (auto& x : w.opvals(j)) sup.push_back(w.supply_of(x));
+      w.reexec[j - p] = 1;
+      w.rx_supply[j] = sup;
+      w.events.push_back({true, j, {P.ins[j].defreg, j}});
+    }
+  Plan pl;
+  pl.valid = true;
+  pl.c = c;
+  pl.p = p;
+  pl.kind = 3;
+  for (int r = 0; r < P.nregs(); r++)
+    if (L.in[p][r]) {
+      pl.saved.push_back({'C', {r, PRE}, -1});
+      (P.is_vec(r) ? pl.n_vec : pl.n_sca)++;
+      pl.payload_bytes += P.is_vec(r) ? VEC_B : SCA_B;
+    }
+  pl.schedule = w.events;
+  pl.reexec_supply = w.rx_supply;
+  for (int r = 0; r < P.nregs(); r++)
+    if (L.in[c][r]) {
+      int d = w.rd(r, c);
+      pl.final_.push_back({r, d == PRE ? Supply{SK::C, -1} : Supply{SK::X, d}});
+    }
+  pl.n_reexec = (uint32_t)w.rx_supply.size();
+  return pl;
+}
+
+Plan window_plan(const Program& P, const Liveness& L, const DefIndex& D, int p, int c, const std::vector<int>& bk,
+                 uint32_t flags) {
+  if (!(flags & F_RELAXED)) return basic_plan(P, L, D, p, c);
+  Window w(P, L, D, p, c, (flags & F_OSRB) ? bk : std::vector<int>{}, flags);
+  w.sweep();
+  if (!w.feasible()) return Plan{};
+  return w.plan(0);
+}
+
+Plan best_plan(const Program& P, const Liveness& L, const DefIndex& D, const std::vector<int>& heads, int c,
+               const std::vector<int>& bk, uint32_t flags) {
+  Plan best;
+  std::vector<int> bc;
+  for (int p = c; p >= heads[c]; p--) {
+    Plan pl = window_plan(P, L, D, p, c, bk, flags);
+    if (!pl.valid) continue;
+    std::vector<int> k = pl.cost();
+    if (!best.valid || k < bc) {
+      best = std::move(pl);
+      bc = k;
+    }
+  }
+  return best;
+}
+
+Plan full_plan(const Program& P, const Liveness& L, int c) {
+  (void)L;
+  Plan pl;
+  pl.valid = true;
+  pl.c = pl.p = c;
+  pl.kind = 2;
+  for (int r = 0; r < P.nregs(); r++) {
+    pl.saved.push_back({'C', {r, PRE}, -1});
+    pl.final_.push_back({r, {SK::C, -1}});
+  }
+  pl.n_vec = P.nv;
+  pl.n_sca = P.ns;
+  pl.payload_bytes = VEC_B * P.nv + SCA_B * P.ns;
+  return pl;
+}
+
+// R-7: irreversible scalar defs whose old value is read in the same BB.
+std::vector<int> osrb_candidates(const Program& P) {
+  std::vector<int> out;
+  for (auto [s, e] : P.bbs)
+    for (int m = s; m < e; m++) {
+      const Instr& I = P.ins[m];
+      int r = I.defreg;
+      if (r < 0 || P.is_vec(r)) continue;
+      RevKind k;
+      std::vector<Operand> oth;
+      if (revert_spec(P, I, r, &k, &oth)) continue;
+      bool read = std::find(I.uses.begin(), I.uses.end(), r) != I.uses.end();
+      for (int j = m - 1; !read && j >= s; j--) {
+        if (P.ins[j].defreg == r) break;
+        if (std::find(P.ins[j].uses.begin(), P.ins[j].uses.end(), r) != P.ins[j].uses.end()) read = true;
+      }
+      if (read) out.push_back(m);
+    }
+  return out;
+}
+
+}  // namespace
+
+std::vector<int> Plan::cost() const {
+  return {(int)payload_bytes, (int)n_rev_pre, (int)(n_reexec + n_rev_res), -p};
+}
+
+Analysis analyze(const Program& P, const Options& opt) {
+  Liveness L = liveness(P);
+  DefIndex D(P);
+  Analysis A;
+  A.live_in = L.in;
+  A.live_out = L.out;
+  A.heads = region_heads(P);
+  A.sites = sites_for(P, opt);
+  A.full_ir_bytes = VEC_B * P.nv + SCA_B * P.ns;
+  for (int c : A.sites) {
+    Window w(P, L, D, c, c, {}, 0);
+    A.live.push_back(w.plan(1));
+  }
+  if (opt.mode == 1) {
+    A.plans = A.live;
+    return A;
+  }
+  if (opt.mode == 2 || opt.mode == 3) {
+    for (int c : A.sites) A.plans.push_back(full_plan(P, L, c));
+    return A;
+  }
+  uint32_t fl = opt.flags;
+  if ((fl & F_OSRB) && (fl & F_RELAXED)) {
+    std::map<int, uint32_t> base;
+    for (int c : A.sites) base[c] = best_plan(P, L, D, A.heads, c, {}, fl).payload_bytes;
+    for (int m : osrb_candidates(P)) {
+      int bbm = P.bb_of[m];
+      for (int c : A.sites) {
+        if (c >= (int)P.ins.size() || P.bb_of[c] != bbm || c <= m || A.heads[c] > m) continue;
+        if (best_plan(P, L, D, A.heads, c, {m}, fl).payload_bytes < base[c]) {
+          A.backups.push_back(m);
+          break;
+        }
+      }
+    }
+  }
+  for (int c : A.sites) A.plans.push_back(best_plan(P, L, D, A.heads, c, A.backups, fl));
+  return A;
+}
+
+// Canonical plan text (identical format to the oracle's plan_text).
+std::string plan_text(const Program& P, const Plan& pl) {
+  auto vs = [&](const Val& v) { return P.regname(v.r) + "@" + (v.d == PRE ? std::string("PRE") : std::to_string(v.d)); };
+  auto ss = [&](const Supply& s) -> std::string {
+    switch (s.k) {
+      case SK::C: return "C";
+      case SK::B: return "B" + std::to_string(s.arg);
+      case SK::X: return "X" + std::to_string(s.arg);
+      case SK::R: return "R" + std::to_string(s.arg);
+    }
+    return "?";
+  };
+  std::ostringstream o;
+  o << "c=" << pl.c << " p=" << pl.p << " bytes=" << pl.payload_bytes << " nv=" << pl.n_vec << " ns=" << pl.n_sca;
+  o << " save=";
+  for (size_t i = 0; i < pl.saved.size(); i++) o << (i ? "," : "") << pl.saved[i].src << ":" << vs(pl.saved[i].v);
+  o << " pre=";
+  for (size_t i = 0; i < pl.pre_reverts.size(); i++)
+    o << (i ? "," : "") << vs(pl.pre_reverts[i].v) << "/m" << pl.pre_reverts[i].m;
+  o << " sched=";
+  for (size_t i = 0; i < pl.schedule.size(); i++) {
+    const Event& e = pl.schedule[i];
+    o << (i ? "," : "");
+    if (e.is_x) {
+      o << "X" << e.j << "(";
+      const auto& sup = pl.reexec_supply.at(e.j);
+      for (size_t k = 0; k < sup.size(); k++) o << (k ? "," : "") << ss(sup[k]);
+      o << ")";
+    } else {
+      const RevertRec& r = pl.revert_info.at(e.v);
+      o << "R" << vs(e.v) << "/m" << r.m << "(";
+      for (size_t k = 0; k < r.supplies.size(); k++) o << (k ? "," : "") << ss(r.supplies[k]);
+      o << ")";
+    }
+  }
+  o << " final=";
+  for (size_t i = 0; i < pl.final_.size(); i++) o << (i ? "," : "") << P.regname(pl.final_[i].first) << ":" << ss(pl.final_[i].second);
+  return o.str();
+}
+
+}  // namespace ctxb

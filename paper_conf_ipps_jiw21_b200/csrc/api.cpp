@@ -1,0 +1,534 @@
+// C ABI of libctxb (include/ctxb.h).  Compile-time part: P:311-317; runtime
+// part: P:319-323 (preemption), P:313-315 (resume).
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <regex>
+
+#include "../../include/ctxb.h"
+#include "ctxb_internal.h"
+#include "driver.h"
+
+using namespace ctxb;
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const std::string& msg) {
+  g_err = msg;
+  return code;
+}
+
+double now_ms() {
+  using namespace std::chrono;
+  return duration<double, std::milli>(steady_clock::now().time_since_epoch()).count();
+}
+
+struct Mod {
+  CUmodule mod = nullptr;
+  CUfunction run = nullptr, resume = nullptr;
+};
+
+std::string cu_err(CUresult r) {
+  const char* s = nullptr;
+  if (driver().ok) driver().cuGetErrorString(r, &s);
+  return s ? s : ("CUresult " + std::to_string((int)r));
+}
+
+#define CU(call)                                                               \
+  do {                                                                         \
+    CUresult _r = (call);                                                      \
+    if (_r != CUDA_SUCCESS) return fail(CTXB_E_CUDA, std::string(#call) + ": " + cu_err(_r)); \
+  } while (0)
+
+}  // namespace
+
+struct ctxb_program {
+  Program prog;
+  Analysis an;
+  Options opt;
+  CodegenInfo cg;
+  std::string src, log;
+  std::vector<char> cubin;
+  uint32_t num_regs = 0;
+  double t_an = 0, t_cg = 0, t_cc = 0;
+  std::mutex mu;
+  std::map<CUcontext, Mod> mods;
+  uint32_t full_ir_words128() const {  // 128-B rows occupied by the FULL_IR layout
+    return (uint32_t)prog.nv + ((uint32_t)prog.ns * 4 + 127) / 128;
+  }
+  uint32_t pad_regs() const {
+    if (opt.mode != CTXB_MODE_FULL_HW) return 0;
+    uint32_t w = full_ir_words128();
+    return num_regs > w ? num_regs - w : 0;
+  }
+  uint32_t full_hw_bytes() const { return (full_ir_words128() + pad_regs()) * 128u; }
+  uint32_t stride() const {
+    uint32_t s = cg.stride;
+    if (opt.mode == CTXB_MODE_FULL_HW) s = std::max(s, full_hw_bytes());
+    return std::max<uint32_t>(128, ((s + 127) / 128) * 128);
+  }
+};
+
+enum { RUN_RUNNING = 0, RUN_PREEMPTED = 1, RUN_DONE = 2 };
+
+struct ctxb_run {
+  ctxb_program* prog = nullptr;
+  CUcontext ctx = nullptr;
+  Mod mod;
+  uint32_t grid = 0, n_warps = 0;
+  std::vector<uint64_t> bufs;
+  std::vector<uint32_t> uni;
+  CUdeviceptr cbuf = 0;
+  uint64_t cbytes = 0, pay_off = 0, stride = 0;
+  CUstream stream = nullptr;
+  CUdeviceptr flag = 0, stamps = 0, forced = 0;
+  uint32_t epoch = 0;
+  int state = RUN_RUNNING;
+  std::vector<uint32_t> hdr_prev, hdr;  // host header snapshots (launch e-1, e)
+  bool resumed_launch = false;
+  ~ctxb_run() {
+    Driver& d = driver();
+    if (d.ok) {
+      if (flag) d.cuMemFree(flag);
+      if (stamps) d.cuMemFree(stamps);
+      if (forced) d.cuMemFree(forced);
+    }
+  }
+};
+
+namespace {
+
+int ensure_ctx(CUcontext* out) {
+  Driver& d = driver();
+  if (!d.ok) return fail(CTXB_E_CUDA, d.err);
+  CUcontext c = nullptr;
+  CU(d.cuCtxGetCurrent(&c));
+  if (!c) {
+    CUdevice dev;
+    CU(d.cuDeviceGet(&dev, 0));
+    CU(d.cuDevicePrimaryCtxRetain(&c, dev));
+    CU(d.cuCtxSetCurrent(c));
+  }
+  *out = c;
+  return CTXB_OK;
+}
+
+int ensure_module(ctxb_program* p, CUcontext c, Mod* out) {
+  if (p->cubin.empty()) return fail(CTXB_E_STATE, "program was analysed with CTXB_DEBUG_NO_COMPILE");
+  std::lock_guard<std::mutex> g(p->mu);
+  auto it = p->mods.find(c);
+  if (it != p->mods.end()) {
+    *out = it->second;
+    return CTXB_OK;
+  }
+  Driver& d = driver();
+  Mod m;
+  CU(d.cuModuleLoadData(&m.mod, p->cubin.data()));
+  CU(d.cuModuleGetFunction(&m.run, m.mod, "ctxb_run"));
+  CU(d.cuModuleGetFunction(&m.resume, m.mod, "ctxb_resume"));
+  int nr = 0;
+  CU(d.cuFuncGetAttribute(&nr, CU_FUNC_ATTRIBUTE_NUM_REGS, m.run));
+  if (p->num_regs == 0) p->num_regs = (uint32_t)nr;
+  p->mods[c] = m;
+  *out = m;
+  return CTXB_OK;
+}
+
+int compile(ctxb_program* p) {
+  Nvrtc& n = nvrtc();
+  if (!n.ok) return fail(CTXB_E_NVRTC, n.err);
+  void* prog = nullptr;
+  int r = n.CreateProgram(&prog, p->src.c_str(), (p->prog.name + ".cu").c_str(), 0, nullptr, nullptr);
+  if (r) return fail(CTXB_E_NVRTC, std::string("nvrtcCreateProgram: ") + n.GetErrorString(r));
+  const char* opts[] = {"--gpu-architecture=sm_100a", "--std=c++17", "-lineinfo", "--fmad=false",
+                        "--ptxas-options=-v", "-DNDEBUG", "-diag-suppress=177,550"};
+  r = n.CompileProgram(prog, (int)(sizeof(opts) / sizeof(opts[0])), opts);
+  size_t ls = 0;
+  n.GetProgramLogSize(prog, &ls);
+  std::string log(ls, '\0');
+  if (ls) n.GetProgramLog(prog, &log[0]);
+  p->log = log;
+  if (r) {
+    n.DestroyProgram(&prog);
+    return fail(CTXB_E_NVRTC, "NVRTC compilation failed: " + log.substr(0, 4000));
+  }
+  size_t cs = 0;
+  n.GetCUBINSize(prog, &cs);
+  p->cubin.resize(cs);
+  n.GetCUBIN(prog, p->cubin.data());
+  n.DestroyProgram(&prog);
+  // ptxas -v: "Compiling entry function 'ctxb_run'" ... "Used N registers"
+  size_t at = log.find("'ctxb_run'");
+  if (at != std::string::npos) {
+    std::smatch m;
+    std::string tail = log.substr(at);
+    if (std::regex_search(tail, m, std::regex("Used ([0-9]+) registers"))) p->num_regs = (uint32_t)std::stoul(m[1]);
+  }
+  return CTXB_OK;
+}
+
+void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>& blob) {
+  size_t nb = std::max<size_t>(1, p->prog.buf_names.size());
+  size_t nu = std::max<size_t>(1, p->prog.uniforms.size());
+  size_t words = nb + 5 + (nu + 4 + 1) / 2;
+  blob.assign(words, 0);
+  for (size_t i = 0; i < r->bufs.size(); i++) blob[i] = r->bufs[i];
+  blob[nb + 0] = r->cbuf;
+  blob[nb + 1] = r->flag;
+  blob[nb + 2] = r->forced;
+  blob[nb + 3] = r->stamps;
+  blob[nb + 4] = r->pay_off;
+  uint32_t* u = reinterpret_cast<uint32_t*>(&blob[nb + 5]);
+  for (size_t i = 0; i < r->uni.size(); i++) u[i] = r->uni[i];
+  u[nu + 0] = r->epoch;
+  u[nu + 1] = (uint32_t)r->stride;
+  u[nu + 2] = p->pad_regs();
+  u[nu + 3] = p->full_hw_bytes();
+}
+
+int upload_forced(ctxb_run* r, const uint32_t* targets) {
+  Driver& d = driver();
+  if (!(r->prog->opt.debug & CTXB_DEBUG_FORCED)) {
+    if (targets) return fail(CTXB_E_INVALID_ARG, "forced_targets given but the program is not CTXB_DEBUG_FORCED");
+    return CTXB_OK;
+  }
+  if (targets) {
+    CU(d.cuMemcpyHtoD(r->forced, targets, (size_t)r->n_warps * 4));
+  } else {
+    CU(d.cuMemsetD32Async(r->forced, 0xFFFFFFFFu, r->n_warps, r->stream));
+  }
+  return CTXB_OK;
+}
+
+int launch(ctxb_run* r, bool resume) {
+  std::vector<uint64_t> blob;
+  pack_params(r, r->prog, blob);
+  void* args[] = {blob.data()};
+  Driver& d = driver();
+  CU(d.cuLaunchKernel(resume ? r->mod.resume : r->mod.run, r->grid, 1, 1, (unsigned)r->prog->prog.block, 1, 1, 0,
+                      r->stream, args, nullptr));
+  r->state = RUN_RUNNING;
+  r->resumed_launch = resume;
+  return CTXB_OK;
+}
+
+// Read the header array after the stream drained and classify the run.
+int collect(ctxb_run* r) {
+  Driver& d = driver();
+  r->hdr_prev.swap(r->hdr);
+  r->hdr.assign((size_t)r->n_warps * 4, 0);
+  CU(d.cuMemcpyDtoH(r->hdr.data(), r->cbuf, (size_t)r->n_warps * 16));
+  uint32_t pre = 0, done = 0;
+  for (uint32_t w = 0; w < r->n_warps; w++) {
+    const uint32_t* h = &r->hdr[(size_t)w * 4];
+    if (h[2] == CTXB_STATE_PREEMPTED && h[3] == r->epoch) pre++;
+    else if (h[2] == CTXB_STATE_DONE) done++;
+  }
+  if (pre + done != r->n_warps)
+    return fail(CTXB_E_CUDA, "kernel did not report every warp (" + std::to_string(pre + done) + "/" +
+                                 std::to_string(r->n_warps) + "): it faulted or was not launched");
+  r->state = pre ? RUN_PREEMPTED : RUN_DONE;
+  return CTXB_OK;
+}
+
+template <class T>
+int copy_out(const std::string& s, T* buf, size_t cap, size_t* len) {
+  if (!len) return fail(CTXB_E_INVALID_ARG, "len is NULL");
+  *len = s.size() + 1;
+  if (!buf || cap < s.size() + 1) return fail(CTXB_E_BUFFER_TOO_SMALL, "buffer too small");
+  memcpy(buf, s.c_str(), s.size() + 1);
+  return CTXB_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* ctxb_last_error(void) { return g_err.c_str(); }
+const char* ctxb_version(void) { return "ctxb 0.1 (sm_100a, CTXB-R1)"; }
+
+int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb_program** out) {
+  if (!ir_text || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  *out = nullptr;
+  ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0};
+  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 7) return fail(CTXB_E_INVALID_ARG, "bad options");
+  std::unique_ptr<ctxb_program> p(new ctxb_program);
+  p->opt = Options{o.flags, o.mode, o.poll_policy, o.poll_every ? o.poll_every : 8, o.debug};
+  try {
+    double t0 = now_ms();
+    p->prog = parse_ir(std::string(ir_text, len));
+    p->an = analyze(p->prog, p->opt);
+    double t1 = now_ms();
+    p->src = generate_cuda(p->prog, p->an, p->opt, &p->cg);
+    double t2 = now_ms();
+    p->t_an = t1 - t0;
+    p->t_cg = t2 - t1;
+  } catch (const ParseError& e) {
+    return fail(CTXB_E_PARSE, e.what());
+  } catch (const std::exception& e) {
+    return fail(CTXB_E_ANALYSIS, std::string("analysis: ") + e.what());
+  }
+  if (!(o.debug & CTXB_DEBUG_NO_COMPILE)) {
+    double t0 = now_ms();
+    int rc = compile(p.get());
+    if (rc) return rc;
+    p->t_cc = now_ms() - t0;
+  }
+  *out = p.release();
+  return CTXB_OK;
+}
+
+int ctxb_program_destroy(ctxb_program* p) {
+  if (!p) return fail(CTXB_E_INVALID_ARG, "NULL program");
+  Driver& d = driver();
+  if (d.ok)
+    for (auto& [c, m] : p->mods) d.cuModuleUnload(m.mod);
+  delete p;
+  return CTXB_OK;
+}
+
+int ctxb_program_info(const ctxb_program* p, ctxb_program_info_t* o) {
+  if (!p || !o) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  o->n_instrs = (uint32_t)p->prog.ins.size();
+  o->nv = (uint32_t)p->prog.nv;
+  o->ns = (uint32_t)p->prog.ns;
+  o->block = (uint32_t)p->prog.block;
+  o->n_buffers = (uint32_t)p->prog.buf_names.size();
+  o->n_uniforms = (uint32_t)p->prog.uniforms.size();
+  o->n_sites = (uint32_t)p->an.sites.size();
+  o->n_backups = (uint32_t)p->an.backups.size();
+  o->max_payload_bytes_per_warp = p->cg.max_payload;
+  o->full_ir_bytes_per_warp = p->an.full_ir_bytes;
+  o->num_regs = p->num_regs;
+  o->compiled = p->cubin.empty() ? 0 : 1;
+  o->analyze_ms = p->t_an;
+  o->codegen_ms = p->t_cg;
+  o->compile_ms = p->t_cc;
+  return CTXB_OK;
+}
+
+int ctxb_num_sites(const ctxb_program* p, uint32_t* n) {
+  if (!p || !n) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  *n = (uint32_t)p->an.sites.size();
+  return CTXB_OK;
+}
+
+int ctxb_site_info(const ctxb_program* p, uint32_t site, ctxb_site_info_t* o) {
+  if (!p || !o) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  if (site >= p->an.sites.size()) return fail(CTXB_E_INVALID_ARG, "site out of range");
+  const Plan& pl = p->an.plans[site];
+  o->c = (uint32_t)pl.c;
+  o->p = (uint32_t)pl.p;
+  o->n_vec = pl.n_vec;
+  o->n_scalar = pl.n_sca;
+  o->n_revert_pre = pl.n_rev_pre;
+  o->n_revert_res = pl.n_rev_res;
+  o->n_reexec = pl.n_reexec;
+  o->payload_bytes_per_warp = pl.payload_bytes;
+  o->live_bytes_per_warp = p->an.live[site].payload_bytes;
+  return CTXB_OK;
+}
+
+int ctxb_backups(const ctxb_program* p, uint32_t* idx, uint32_t cap, uint32_t* n) {
+  if (!p || !n) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  *n = (uint32_t)p->an.backups.size();
+  for (uint32_t i = 0; i < *n && i < cap && idx; i++) idx[i] = (uint32_t)p->an.backups[i];
+  return CTXB_OK;
+}
+
+int ctxb_site_plan_text(const ctxb_program* p, uint32_t site, int live, char* buf, size_t cap, size_t* len) {
+  if (!p) return fail(CTXB_E_INVALID_ARG, "NULL program");
+  if (site >= p->an.sites.size()) return fail(CTXB_E_INVALID_ARG, "site out of range");
+  return copy_out(plan_text(p->prog, live ? p->an.live[site] : p->an.plans[site]), buf, cap, len);
+}
+
+int ctxb_generated_source(const ctxb_program* p, char* buf, size_t cap, size_t* len) {
+  if (!p) return fail(CTXB_E_INVALID_ARG, "NULL program");
+  return copy_out(p->src, buf, cap, len);
+}
+
+int ctxb_context_capacity(const ctxb_program* p, uint32_t grid, uint64_t* bytes) {
+  if (!p || !bytes || grid == 0) return fail(CTXB_E_INVALID_ARG, "bad argument");
+  if (p->opt.mode == CTXB_MODE_FULL_HW && p->num_regs == 0)
+    return fail(CTXB_E_STATE, "FULL_HW capacity needs the compiled register count");
+  uint64_t nw = (uint64_t)grid * (p->prog.block / 32);
+  uint64_t off = ((nw * 16 + 255) / 256) * 256;
+  *bytes = off + nw * p->stride();
+  return CTXB_OK;
+}
+
+int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint32_t* uniforms, void* ctx_buf,
+                uint64_t ctx_bytes, void* stream, const uint32_t* forced_targets, ctxb_run** out) {
+  if (!p || !out || grid == 0) return fail(CTXB_E_INVALID_ARG, "bad argument");
+  *out = nullptr;
+  if (!p->prog.buf_names.empty() && !buffers) return fail(CTXB_E_INVALID_ARG, "buffers is NULL");
+  if (!p->prog.uniforms.empty() && !uniforms) return fail(CTXB_E_INVALID_ARG, "uniforms is NULL");
+  if (!ctx_buf) return fail(CTXB_E_INVALID_ARG, "ctx_buf is NULL");
+  CUcontext c;
+  int rc = ensure_ctx(&c);
+  if (rc) return rc;
+  std::unique_ptr<ctxb_run> r(new ctxb_run);
+  r->prog = p;
+  r->ctx = c;
+  rc = ensure_module(p, c, &r->mod);
+  if (rc) return rc;
+  uint64_t need = 0;
+  rc = ctxb_context_capacity(p, grid, &need);
+  if (rc) return rc;
+  if (ctx_bytes < need)
+    return fail(CTXB_E_BUFFER_TOO_SMALL, "context buffer has " + std::to_string(ctx_bytes) + " bytes, needs " +
+                                             std::to_string(need));
+  Driver& d = driver();
+  r->grid = grid;
+  r->n_warps = grid * (p->prog.block / 32);
+  for (size_t i = 0; i < p->prog.buf_names.size(); i++) r->bufs.push_back((uint64_t)(uintptr_t)buffers[i]);
+  for (size_t i = 0; i < p->prog.uniforms.size(); i++) r->uni.push_back(uniforms[i]);
+  r->cbuf = (CUdeviceptr)(uintptr_t)ctx_buf;
+  r->cbytes = ctx_bytes;
+  r->pay_off = (((uint64_t)r->n_warps * 16 + 255) / 256) * 256;
+  r->stride = p->stride();
+  r->stream = (CUstream)stream;
+  CU(d.cuMemAlloc(&r->flag, 256));
+  CU(d.cuMemAlloc(&r->stamps, (size_t)r->n_warps * 32));
+  CU(d.cuMemAlloc(&r->forced, (size_t)r->n_warps * 4));
+  CU(d.cuMemsetD32Async(r->flag, 0, 64, r->stream));
+  CU(d.cuMemsetD32Async(r->stamps, 0, (size_t)r->n_warps * 8, r->stream));
+  CU(d.cuMemsetD32Async(r->cbuf, 0, (size_t)r->n_warps * 4, r->stream));   // headers
+  rc = upload_forced(r.get(), forced_targets);
+  if (rc) return rc;
+  r->epoch = 1;
+  rc = launch(r.get(), false);
+  if (rc) return rc;
+  *out = r.release();
+  return CTXB_OK;
+}
+
+int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
+  if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
+  if (r->state != RUN_RUNNING) return fail(CTXB_E_STATE, "run is not running");
+  if ((CUstream)ctrl == r->stream && ctrl != nullptr)
+    return fail(CTXB_E_INVALID_ARG, "ctrl_stream must differ from the run's stream");
+  Driver& d = driver();
+  double t0 = now_ms();
+  CU(d.cuStreamWriteValue32((CUstream)ctrl, r->flag, 1u, 0));
+  CU(d.cuStreamSynchronize(r->stream));
+  double t1 = now_ms();
+  CU(d.cuMemsetD32Async(r->flag, 0, 1, (CUstream)ctrl));
+  CU(d.cuStreamSynchronize((CUstream)ctrl));
+  int rc = collect(r);
+  if (rc) return rc;
+  if (st) {
+    memset(st, 0, sizeof *st);
+    st->host_us = (t1 - t0) * 1e3;
+    std::vector<uint64_t> stamps((size_t)r->n_warps * 4);
+    CU(d.cuMemcpyDtoH(stamps.data(), r->stamps, stamps.size() * 8));
+    uint64_t tmin = UINT64_MAX, tmax = 0;
+    std::vector<uint8_t> blk(r->grid, 0);
+    uint32_t nwb = r->prog->prog.block / 32;
+    for (uint32_t w = 0; w < r->n_warps; w++) {
+      const uint32_t* h = &r->hdr[(size_t)w * 4];
+      if (h[2] == CTXB_STATE_PREEMPTED && h[3] == r->epoch) {
+        st->warps_preempted++;
+        st->payload_bytes += h[1];
+        st->header_bytes += 16;
+        blk[w / nwb] = 1;
+        tmin = std::min(tmin, stamps[(size_t)w * 4 + 0]);
+        tmax = std::max(tmax, stamps[(size_t)w * 4 + 1]);
+      } else if (h[2] == CTXB_STATE_DONE) {
+        st->warps_done++;
+      }
+    }
+    for (auto b : blk) st->blocks_preempted += b;
+    st->latency_us = st->warps_preempted ? (double)(tmax - tmin) * 1e-3 : 0.0;
+  }
+  return CTXB_OK;
+}
+
+int ctxb_resume(ctxb_run* r, void* stream, const uint32_t* forced_targets) {
+  if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
+  if (r->state != RUN_PREEMPTED) return fail(CTXB_E_STATE, "run is not preempted");
+  r->stream = (CUstream)stream;
+  int rc = upload_forced(r, forced_targets);
+  if (rc) return rc;
+  r->epoch++;
+  return launch(r, true);
+}
+
+int ctxb_wait(ctxb_run* r, int* finished) {
+  if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
+  if (r->state == RUN_RUNNING) {
+    CU(driver().cuStreamSynchronize(r->stream));
+    int rc = collect(r);
+    if (rc) return rc;
+  }
+  if (finished) *finished = r->state == RUN_DONE ? 1 : 0;
+  return CTXB_OK;
+}
+
+int ctxb_resume_stats_get(const ctxb_run* r, ctxb_resume_stats* o) {
+  if (!r || !o) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  memset(o, 0, sizeof *o);
+  if (!r->resumed_launch || r->state == RUN_RUNNING || r->hdr_prev.empty()) return CTXB_OK;
+  std::vector<uint64_t> stamps((size_t)r->n_warps * 4);
+  CU(driver().cuMemcpyDtoH(stamps.data(), r->stamps, stamps.size() * 8));
+  uint64_t tmin = UINT64_MAX, tmax = 0;
+  for (uint32_t w = 0; w < r->n_warps; w++) {
+    const uint32_t* h = &r->hdr_prev[(size_t)w * 4];
+    if (h[2] == CTXB_STATE_PREEMPTED && h[3] + 1 == r->epoch) {
+      o->warps_resumed++;
+      tmin = std::min(tmin, stamps[(size_t)w * 4 + 2]);
+      tmax = std::max(tmax, stamps[(size_t)w * 4 + 3]);
+    }
+  }
+  o->resume_us = o->warps_resumed ? (double)(tmax - tmin) * 1e-3 : 0.0;
+  return CTXB_OK;
+}
+
+int ctxb_context_bytes(const ctxb_run* r, uint64_t* payload, uint64_t* header, uint32_t* n_tb) {
+  if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
+  uint64_t pb = 0, hb = 0;
+  uint32_t nwb = r->prog->prog.block / 32;
+  std::vector<uint8_t> blk(r->grid, 0);
+  for (uint32_t w = 0; w < r->n_warps && !r->hdr.empty(); w++) {
+    const uint32_t* h = &r->hdr[(size_t)w * 4];
+    if (h[2] == CTXB_STATE_PREEMPTED && h[3] == r->epoch) {
+      pb += h[1];
+      hb += 16;
+      blk[w / nwb] = 1;
+    }
+  }
+  uint32_t nt = 0;
+  for (auto b : blk) nt += b;
+  if (payload) *payload = pb;
+  if (header) *header = hb;
+  if (n_tb) *n_tb = nt;
+  return CTXB_OK;
+}
+
+int ctxb_read_headers(const ctxb_run* r, uint32_t* out, uint64_t n) {
+  if (!r || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  if (n < (uint64_t)r->n_warps * 4) return fail(CTXB_E_BUFFER_TOO_SMALL, "need 4 words per warp");
+  if (r->hdr.empty()) return fail(CTXB_E_STATE, "no completed launch yet");
+  memcpy(out, r->hdr.data(), (size_t)r->n_warps * 16);
+  return CTXB_OK;
+}
+
+int ctxb_read_stamps(const ctxb_run* r, uint64_t* out, uint64_t n) {
+  if (!r || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  if (n < (uint64_t)r->n_warps * 4) return fail(CTXB_E_BUFFER_TOO_SMALL, "need 4 words per warp");
+  CU(driver().cuMemcpyDtoH(out, r->stamps, (size_t)r->n_warps * 32));
+  return CTXB_OK;
+}
+
+int ctxb_run_destroy(ctxb_run* r) {
+  if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
+  delete r;
+  return CTXB_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,293 @@
+"""ctypes binding of libctxb (include/ctxb.h) -- argument marshalling only.
+
+Every function named ``ctxb_*`` here calls the C entry point of the same name
+(the boundary, include/ctxb.h); ``Program`` and ``Run`` are thin handle
+wrappers over them.  Device memory and streams come from the caller (torch
+tensors / streams, or raw integers); nothing is computed here.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+__all__ = [
+    "LIB_PATH", "CtxbError", "lib",
+    "RELAXED", "REVERT", "OSRB", "ALL", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
+    "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
+    "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE",
+    "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "EXPORTED_SYMBOLS",
+    "ctxb_analyze", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait", "ctxb_context_bytes",
+    "Program", "Run",
+]
+
+LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libctxb.so")
+
+RELAXED, REVERT, OSRB, ALL = 1, 2, 4, 7
+MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
+POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
+DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE = 1, 2, 4, 8
+STATE_NONE, STATE_PREEMPTED, STATE_DONE = 0, 1, 2
+NEVER = 0xFFFFFFFF
+
+EXPORTED_SYMBOLS = [
+    "ctxb_last_error", "ctxb_version", "ctxb_analyze", "ctxb_program_destroy", "ctxb_program_info",
+    "ctxb_num_sites", "ctxb_site_info", "ctxb_backups", "ctxb_site_plan_text", "ctxb_generated_source",
+    "ctxb_context_capacity", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait",
+    "ctxb_resume_stats_get", "ctxb_context_bytes", "ctxb_read_headers", "ctxb_read_stamps",
+    "ctxb_run_destroy",
+]
+
+
+class CtxbError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"ctxb error {code}: {msg}")
+        self.code = code
+
+
+class _Opts(C.Structure):
+    _fields_ = [("flags", C.c_uint32), ("mode", C.c_uint32), ("poll_policy", C.c_uint32),
+                ("poll_every", C.c_uint32), ("debug", C.c_uint32)]
+
+
+class _SiteInfo(C.Structure):
+    _fields_ = [(n, C.c_uint32) for n in ("c", "p", "n_vec", "n_scalar", "n_revert_pre", "n_revert_res",
+                                          "n_reexec", "payload_bytes_per_warp", "live_bytes_per_warp")]
+
+
+class _ProgInfo(C.Structure):
+    _fields_ = [(n, C.c_uint32) for n in ("n_instrs", "nv", "ns", "block", "n_buffers", "n_uniforms", "n_sites",
+                                          "n_backups", "max_payload_bytes_per_warp", "full_ir_bytes_per_warp",
+                                          "num_regs", "compiled")] + \
+               [("analyze_ms", C.c_double), ("codegen_ms", C.c_double), ("compile_ms", C.c_double)]
+
+
+class _PreStats(C.Structure):
+    _fields_ = [("latency_us", C.c_double), ("host_us", C.c_double), ("warps_preempted", C.c_uint32),
+                ("warps_done", C.c_uint32), ("blocks_preempted", C.c_uint32), ("payload_bytes", C.c_uint64),
+                ("header_bytes", C.c_uint64)]
+
+
+class _ResStats(C.Structure):
+    _fields_ = [("resume_us", C.c_double), ("warps_resumed", C.c_uint32)]
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"libctxb.so not built ({LIB_PATH}); run __graft_entry__.build() -- "
+                          "there is no CPU fallback")
+    L = C.CDLL(LIB_PATH)
+    P, U32, U64, SZ, I = C.c_void_p, C.c_uint32, C.c_uint64, C.c_size_t, C.c_int
+    sig = {
+        "ctxb_last_error": (C.c_char_p, []),
+        "ctxb_version": (C.c_char_p, []),
+        "ctxb_analyze": (I, [C.c_char_p, SZ, C.POINTER(_Opts), C.POINTER(P)]),
+        "ctxb_program_destroy": (I, [P]),
+        "ctxb_program_info": (I, [P, C.POINTER(_ProgInfo)]),
+        "ctxb_num_sites": (I, [P, C.POINTER(U32)]),
+        "ctxb_site_info": (I, [P, U32, C.POINTER(_SiteInfo)]),
+        "ctxb_backups": (I, [P, C.POINTER(U32), U32, C.POINTER(U32)]),
+        "ctxb_site_plan_text": (I, [P, U32, I, C.c_char_p, SZ, C.POINTER(SZ)]),
+        "ctxb_generated_source": (I, [P, C.c_char_p, SZ, C.POINTER(SZ)]),
+        "ctxb_context_capacity": (I, [P, U32, C.POINTER(U64)]),
+        "ctxb_launch": (I, [P, U32, C.POINTER(P), C.POINTER(U32), P, U64, P, C.POINTER(U32), C.POINTER(P)]),
+        "ctxb_preempt": (I, [P, P, C.POINTER(_PreStats)]),
+        "ctxb_resume": (I, [P, P, C.POINTER(U32)]),
+        "ctxb_wait": (I, [P, C.POINTER(I)]),
+        "ctxb_resume_stats_get": (I, [P, C.POINTER(_ResStats)]),
+        "ctxb_context_bytes": (I, [P, C.POINTER(U64), C.POINTER(U64), C.POINTER(U32)]),
+        "ctxb_read_headers": (I, [P, C.POINTER(U32), U64]),
+        "ctxb_read_stamps": (I, [P, C.POINTER(U64), U64]),
+        "ctxb_run_destroy": (I, [P]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    return L
+
+
+lib = _load()
+
+
+def _chk(rc):
+    if rc != 0:
+        raise CtxbError(rc, lib.ctxb_last_error().decode(errors="replace"))
+
+
+def _ptr(x):
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    return int(x.data_ptr())
+
+
+def _stream(s):
+    if s is None:
+        return None
+    if isinstance(s, int):
+        return s
+    return int(s.cuda_stream)
+
+
+def _u32arr(vals):
+    if vals is None:
+        return None
+    a = np.ascontiguousarray(np.asarray(vals, dtype=np.uint32))
+    return a, a.ctypes.data_as(C.POINTER(C.c_uint32))
+
+
+# --- the C-ABI names ----------------------------------------------------------
+
+def ctxb_analyze(ir_text: str, flags=ALL, mode=MODE_CTXBACK, poll_policy=POLL_EVERY_INSTR, poll_every=8,
+                 debug=0) -> "Program":
+    return Program(ir_text, flags, mode, poll_policy, poll_every, debug)
+
+
+def ctxb_launch(prog, grid, buffers, uniforms, ctx, stream=None, forced=None) -> "Run":
+    return prog.launch(grid, buffers, uniforms, ctx, stream, forced)
+
+
+def ctxb_preempt(run, ctrl_stream):
+    return run.preempt(ctrl_stream)
+
+
+def ctxb_resume(run, stream=None, forced=None):
+    return run.resume(stream, forced)
+
+
+def ctxb_wait(run):
+    return run.wait()
+
+
+def ctxb_context_bytes(run):
+    return run.context_bytes()
+
+
+class Program:
+    """An analysed + compiled IR kernel (ctxb_analyze)."""
+
+    def __init__(self, ir_text, flags=ALL, mode=MODE_CTXBACK, poll_policy=POLL_EVERY_INSTR, poll_every=8,
+                 debug=0):
+        self._h = C.c_void_p()
+        o = _Opts(flags, mode, poll_policy, poll_every, debug)
+        b = ir_text.encode()
+        _chk(lib.ctxb_analyze(b, len(b), C.byref(o), C.byref(self._h)))
+        self.debug = debug
+
+    def __del__(self):
+        if getattr(self, "_h", None):
+            lib.ctxb_program_destroy(self._h)
+            self._h = None
+
+    @property
+    def info(self):
+        i = _ProgInfo()
+        _chk(lib.ctxb_program_info(self._h, C.byref(i)))
+        return {k: getattr(i, k) for k, _ in _ProgInfo._fields_}
+
+    @property
+    def num_sites(self):
+        n = C.c_uint32()
+        _chk(lib.ctxb_num_sites(self._h, C.byref(n)))
+        return n.value
+
+    def site_info(self, k):
+        s = _SiteInfo()
+        _chk(lib.ctxb_site_info(self._h, k, C.byref(s)))
+        return {n: getattr(s, n) for n, _ in _SiteInfo._fields_}
+
+    @property
+    def backups(self):
+        n = C.c_uint32()
+        _chk(lib.ctxb_backups(self._h, None, 0, C.byref(n)))
+        a = (C.c_uint32 * max(1, n.value))()
+        _chk(lib.ctxb_backups(self._h, a, n.value, C.byref(n)))
+        return [a[i] for i in range(n.value)]
+
+    def _text(self, fn, *args):
+        ln = C.c_size_t()
+        rc = fn(self._h, *args, None, 0, C.byref(ln))
+        if rc not in (0, -7):
+            _chk(rc)
+        buf = C.create_string_buffer(ln.value)
+        _chk(fn(self._h, *args, buf, ln.value, C.byref(ln)))
+        return buf.value.decode()
+
+    def plan_text(self, k, live=False):
+        return self._text(lib.ctxb_site_plan_text, k, 1 if live else 0)
+
+    @property
+    def source(self):
+        return self._text(lib.ctxb_generated_source)
+
+    def context_capacity(self, grid):
+        b = C.c_uint64()
+        _chk(lib.ctxb_context_capacity(self._h, grid, C.byref(b)))
+        return b.value
+
+    def launch(self, grid, buffers, uniforms, ctx, stream=None, forced=None, ctx_bytes=None):
+        bufs = (C.c_void_p * max(1, len(buffers)))(*[_ptr(b) for b in buffers])
+        uni = _u32arr(uniforms if uniforms else [0])
+        f = _u32arr(forced)
+        if ctx_bytes is None:
+            ctx_bytes = ctx.numel() * ctx.element_size() if hasattr(ctx, "numel") else 0
+        h = C.c_void_p()
+        _chk(lib.ctxb_launch(self._h, grid, bufs, uni[1], _ptr(ctx), ctx_bytes, _stream(stream),
+                             f[1] if f else None, C.byref(h)))
+        return Run(h, self, grid, (buffers, ctx))
+
+
+class Run:
+    """One launch and its preempt / resume history (ctxb_launch)."""
+
+    def __init__(self, h, prog, grid, keep):
+        self._h = h
+        self.prog = prog
+        self.grid = grid
+        self._keep = keep          # keep the caller's tensors alive
+
+    def __del__(self):
+        if getattr(self, "_h", None):
+            lib.ctxb_run_destroy(self._h)
+            self._h = None
+
+    @property
+    def n_warps(self):
+        return self.grid * self.prog.info["block"] // 32
+
+    def preempt(self, ctrl_stream):
+        s = _PreStats()
+        _chk(lib.ctxb_preempt(self._h, _stream(ctrl_stream), C.byref(s)))
+        return {k: getattr(s, k) for k, _ in _PreStats._fields_}
+
+    def resume(self, stream=None, forced=None):
+        f = _u32arr(forced)
+        _chk(lib.ctxb_resume(self._h, _stream(stream), f[1] if f else None))
+
+    def wait(self):
+        fin = C.c_int()
+        _chk(lib.ctxb_wait(self._h, C.byref(fin)))
+        return bool(fin.value)
+
+    def resume_stats(self):
+        s = _ResStats()
+        _chk(lib.ctxb_resume_stats_get(self._h, C.byref(s)))
+        return {k: getattr(s, k) for k, _ in _ResStats._fields_}
+
+    def context_bytes(self):
+        p, h, n = C.c_uint64(), C.c_uint64(), C.c_uint32()
+        _chk(lib.ctxb_context_bytes(self._h, C.byref(p), C.byref(h), C.byref(n)))
+        return p.value, h.value, n.value
+
+    def headers(self):
+        a = np.zeros(self.n_warps * 4, dtype=np.uint32)
+        _chk(lib.ctxb_read_headers(self._h, a.ctypes.data_as(C.POINTER(C.c_uint32)), a.size))
+        return a.reshape(-1, 4)
+
+    def stamps(self):
+        a = np.zeros(self.n_warps * 4, dtype=np.uint64)
+        _chk(lib.ctxb_read_stamps(self._h, a.ctypes.data_as(C.POINTER(C.c_uint64)), a.size))
+        return a.reshape(-1, 4)

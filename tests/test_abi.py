@@ -1,0 +1,112 @@
+"""CPU tests of the C-ABI library: it loads without a GPU, exports every
+symbol include/ctxb.h declares, reports errors through status codes, and its
+analyzer (C++, independent of the oracle) produces plans identical to the
+oracle's on random programs and the configs (parity of the compile-time
+part, runs without a GPU)."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_ipps_jiw21_b200 as cb
+from oracle import analysis as A
+from oracle import ir
+from workloads import configs
+from workloads.randprog import random_program
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_symbols():
+    txt = open(os.path.join(ROOT, "include", "ctxb.h")).read()
+    return sorted(set(re.findall(r"\b(ctxb_[a-z_]+)\s*\(", txt)))
+
+
+def test_library_exports_every_header_symbol():
+    lib = ctypes.CDLL(cb.LIB_PATH)
+    syms = header_symbols()
+    assert len(syms) >= 19
+    for s in syms:
+        assert hasattr(lib, s), s
+    assert sorted(cb.EXPORTED_SYMBOLS) == syms
+
+
+def test_parse_errors_are_status_codes():
+    bad = [".kernel k\n.vregs 1\n.sregs 0\n.block 32\n  bogus v0\n  exit\n",
+           ".kernel k\n.vregs 1\n.sregs 0\n.block 33\n  exit\n",
+           ".kernel k\n.vregs 1\n.sregs 1\n.block 32\n  mov s0, %tid\n  exit\n",
+           ".kernel k\n.vregs 1\n.sregs 0\n.block 32\n  mov v3, 1\n  exit\n",
+           ".kernel k\n.vregs 1\n.sregs 0\n.block 32\n  mov v0, 1\n"]
+    for t in bad:
+        with pytest.raises(cb.CtxbError) as e:
+            cb.Program(t, debug=cb.DEBUG_NO_COMPILE)
+        assert e.value.code == -2
+        with pytest.raises(ir.IRError):
+            ir.parse(t)
+
+
+def test_gpu_calls_fail_loudly_without_device():
+    try:
+        import torch
+        if torch.cuda.is_available():
+            pytest.skip("a GPU is present")
+    except Exception:
+        pass
+    p = cb.Program(configs.c1()["ir"], debug=cb.DEBUG_NO_COMPILE)
+    with pytest.raises(cb.CtxbError):
+        p.launch(1, [1, 2, 3, 4], [], 5, ctx_bytes=1 << 20)
+
+
+def _same_plans(txt, policy="EVERY_INSTR", flags=7, mode=0):
+    op = ir.parse(txt)
+    an = A.analyze(op, policy=policy, flags=flags, mode=mode)
+    pol = {"EVERY_INSTR": 0, "EVERY_N": 1, "EXPLICIT": 2}[policy]
+    p = cb.Program(txt, flags=flags, mode=mode, poll_policy=pol, debug=cb.DEBUG_NO_COMPILE)
+    assert p.num_sites == len(an.sites)
+    assert p.backups == an.backups
+    for k, c in enumerate(an.sites):
+        assert p.plan_text(k) == A.plan_text(op, an.plans[c]), (k, c)
+        assert p.plan_text(k, live=True) == A.plan_text(op, an.live[c])
+        si = p.site_info(k)
+        assert (si["c"], si["p"], si["payload_bytes_per_warp"]) == (c, an.plans[c].p, an.plans[c].payload_bytes)
+        assert si["live_bytes_per_warp"] == an.live[c].payload_bytes
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_analyzer_parity_random(seed):
+    txt, _ = random_program(seed, loop=seed % 3 == 0, n_body=10)
+    _same_plans(txt)
+
+
+@pytest.mark.parametrize("flags", [0, 1, 3, 5, 7])
+def test_analyzer_parity_technique_toggles(flags):
+    for seed in range(8):
+        txt, _ = random_program(100 + seed, loop=seed % 2 == 0, n_body=9)
+        _same_plans(txt, flags=flags)
+
+
+@pytest.mark.parametrize("mode", [1, 2])
+def test_analyzer_parity_live_full(mode):
+    txt, _ = random_program(7, loop=True, n_body=9)
+    _same_plans(txt, mode=mode)
+
+
+def test_analyzer_parity_c1():
+    _same_plans(configs.c1()["ir"])
+
+
+def test_analyzer_parity_every_n():
+    for seed in range(6):
+        txt, _ = random_program(200 + seed, loop=True, n_body=14)
+        _same_plans(txt, policy="EVERY_N")
+
+
+def test_context_capacity_layout():
+    p = cb.Program(configs.c1()["ir"], debug=cb.DEBUG_NO_COMPILE)
+    info = p.info
+    stride = ((info["max_payload_bytes_per_warp"] + 127) // 128) * 128
+    for grid in (1, 7, 148):
+        nw = grid * 4
+        assert p.context_capacity(grid) == ((nw * 16 + 255) // 256) * 256 + nw * max(128, stride)

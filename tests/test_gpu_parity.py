@@ -1,0 +1,112 @@
+"""GPU parity: the generated sm_100a kernels (through the C-ABI) against the
+oracle, on the same seeded inputs, element by element.
+
+* uninterrupted outputs are bit-exact with the oracle interpreter;
+* forced preemption at every site / random per-warp sites / nested
+  re-preemption: final outputs bit-exact with the uninterrupted run and the
+  oracle, and every preempted warp's header (site, LIVE-fallback flag,
+  payload bytes) equals the oracle's record (context bytes == oracle's);
+* the same with the poison debug mode (every IR register of a resumed warp
+  starts as garbage, so a plan that relies on an unsaved register fails).
+"""
+import numpy as np
+import pytest
+
+from oracle import analysis as A
+from oracle import interp, ir
+from workloads import configs
+from workloads.randprog import random_buffers, random_program
+
+from gpu_helpers import gpu_run, header_records, oracle_records
+
+pytestmark = pytest.mark.gpu
+
+
+def _cb():
+    import paper_conf_ipps_jiw21_b200 as cb
+    return cb
+
+
+def check(txt, grid, bufs, schedules, policy="EVERY_INSTR", skip=("scr",), poison=True, flags=7):
+    cb = _cb()
+    op = ir.parse(txt)
+    an = A.analyze(op, policy=policy, flags=flags)
+    pol = {"EVERY_INSTR": cb.POLL_EVERY_INSTR, "EXPLICIT": cb.POLL_EXPLICIT}[policy]
+    dbg = cb.DEBUG_FORCED | (cb.DEBUG_POISON if poison else 0)
+    prog = cb.Program(txt, flags=flags, poll_policy=pol, debug=dbg)
+    names = list(op.buffers)
+    ref, _ = interp.run(an, grid, bufs)
+    g0, h0, _ = gpu_run(prog, names, grid, bufs, {})
+    for n in names:
+        if n in skip:
+            continue
+        assert np.array_equal(g0[n], ref[n]), f"uninterrupted output {n} differs from the oracle"
+    for sched in schedules:
+        out, rec = interp.run(an, grid, bufs, schedule=sched)
+        g, hdrs, run = gpu_run(prog, names, grid, bufs, {}, schedule=sched)
+        for n in names:
+            if n in skip:
+                continue
+            assert np.array_equal(g[n], ref[n]), f"{n} after preempt/resume differs (schedule {sched})"
+            assert np.array_equal(out[n], ref[n])
+        assert header_records(hdrs) [:len(oracle_records(rec, an))] == oracle_records(rec, an)
+    return prog, an
+
+
+def test_c1_every_site_all_warps():
+    cfg = configs.c1()
+    scheds = [[[k] * 4] for k in range(24)]
+    check(cfg["ir"], 1, cfg["buffers"], scheds)
+
+
+def test_c1_random_per_warp_sites_and_nested():
+    cfg = configs.c1()
+    vecs = configs.c1_random_site_vectors(512)
+    r = np.random.default_rng(8)
+    scheds = []
+    for i, v in enumerate(vecs):
+        if i % 4 == 0:   # nested: re-preempt after the resume (LIVE fallback in the same BB pass)
+            scheds.append([v, r.integers(0, 6, 4).astype(np.uint32)])
+        else:
+            scheds.append([v])
+    check(cfg["ir"], 1, cfg["buffers"], scheds)
+
+
+def test_c1_bytes_equal_oracle_per_site():
+    cb = _cb()
+    cfg = configs.c1()
+    op = ir.parse(cfg["ir"])
+    an = A.analyze(op)
+    prog = cb.Program(cfg["ir"], debug=cb.DEBUG_NO_COMPILE)
+    for k, c in enumerate(an.sites):
+        si = prog.site_info(k)
+        assert si["payload_bytes_per_warp"] == an.plans[c].payload_bytes
+        assert si["p"] == an.plans[c].p
+        assert prog.plan_text(k) == A.plan_text(op, an.plans[c])
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_random_programs(seed):
+    loop = seed % 3 == 0
+    txt, size = random_program(seed, loop=loop, n_body=10)
+    op = ir.parse(txt)
+    grid = 3
+    nout = op.nv - 1 + op.ns - (1 if loop else 0)
+    bufs = random_buffers(seed, op.block, grid, size, nout)
+    r = np.random.default_rng(seed)
+    nw = grid * op.nwarps
+    scheds = [[r.integers(0, 60, nw).astype(np.uint32), r.integers(0, 20, nw).astype(np.uint32)] for _ in range(6)]
+    check(txt, grid, bufs, scheds)
+
+
+@pytest.mark.parametrize("name", ["fig2", "fig3", "fig4", "fig5", "fig6", "r9"])
+def test_paper_figures_on_gpu(name):
+    import json
+    import os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", name + ".json")))
+    op = ir.parse(g["ir"])
+    r = np.random.default_rng(3)
+    bufs = {b: (r.integers(0, 64, 64, dtype=np.uint32) if k == "ro" else np.zeros(64, np.uint32))
+            for b, k in op.buffers.items()}
+    n = len(op.instrs)
+    check(g["ir"], 1, bufs, [[[k]] for k in range(n)])
