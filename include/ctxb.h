@@ -88,6 +88,13 @@ typedef struct {
   uint32_t poll_policy; /* CTXB_POLL_*                                           */
   uint32_t poll_every;  /* N for CTXB_POLL_EVERY_N                               */
   uint32_t debug;       /* CTXB_DEBUG_* bits                                     */
+  uint32_t flag_depth;  /* flag-load pipeline depth D >= 1 (0 = 1): a poll site
+                           tests the flag value loaded D sites earlier, hiding the
+                           L2 round trip behind D site intervals (dense sites ->
+                           larger D)                                              */
+  uint32_t min_blocks_per_sm; /* 0 = compiler's choice; else both generated kernels
+                           get __launch_bounds__(block, n): ptxas caps registers
+                           so n blocks fit per SM (persistent-grid occupancy)      */
 } ctxb_options;
 
 typedef struct ctxb_program ctxb_program; /* analysed IR kernel + module; library-owned */
@@ -112,6 +119,10 @@ typedef struct {
   uint32_t full_ir_bytes_per_warp;     /* 128*nv + 4*ns                              */
   uint32_t num_regs;                   /* ptxas registers/thread (0 if not compiled) */
   uint32_t compiled;                   /* 1 if a cubin was produced                  */
+  uint32_t num_regs_resume;            /* ptxas registers/thread of the resume kernel */
+  uint32_t resume_maxnreg;             /* min blocks/SM requested for the resume kernel
+                                          (__launch_bounds__) so it keeps the normal
+                                          kernel's occupancy (0 = none needed)       */
   double analyze_ms, codegen_ms, compile_ms;
 } ctxb_program_info_t;
 
@@ -135,7 +146,7 @@ const char* ctxb_version(void);
 
 /* Parse + analyse + generate + compile.  `ir_text` need not be
  * NUL-terminated (`len` bytes are read).  opts == NULL means
- * {CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0}.
+ * {CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0}.
  * Errors: _INVALID_ARG, _PARSE, _ANALYSIS, _NVRTC. */
 int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb_program** out);
 int ctxb_program_destroy(ctxb_program* prog);
@@ -150,6 +161,12 @@ int ctxb_site_plan_text(const ctxb_program* prog, uint32_t site, int live, char*
                         size_t* len);
 /* The generated CUDA C++ source (same buffer convention). */
 int ctxb_generated_source(const ctxb_program* prog, char* buf, size_t cap, size_t* len);
+
+/* Resident blocks per SM of the generated kernels (min over the normal and the
+ * resume kernel, driver occupancy calculator) and the device's SM count: a
+ * persistent grid is blocks_per_sm * num_sms ("persistent thread").
+ * Needs a GPU (_CUDA otherwise). */
+int ctxb_occupancy(ctxb_program* prog, uint32_t* blocks_per_sm, uint32_t* num_sms);
 
 /* Bytes of device memory a context buffer for `grid_blocks` blocks needs:
  * 16 B header per warp + per-warp payload slots. */
@@ -181,6 +198,11 @@ int ctxb_resume(ctxb_run* run, void* stream, const uint32_t* forced_targets);
 /* Wait for the run's current launch; *finished = 1 if every warp is done,
  * 0 if some warps were preempted (forced mode or a racing ctxb_preempt). */
 int ctxb_wait(ctxb_run* run, int* finished);
+
+/* Duration of the run's last kernel launch (normal or resume), from CUDA
+ * events the library records immediately before and after cuLaunchKernel on
+ * the launching stream.  Valid after ctxb_wait / ctxb_preempt returned. */
+int ctxb_launch_ms(const ctxb_run* run, float* ms);
 
 /* Device timings of the last resume launch (valid after ctxb_wait/preempt). */
 int ctxb_resume_stats_get(const ctxb_run* run, ctxb_resume_stats* out);

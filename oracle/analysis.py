@@ -25,6 +25,7 @@ on entry to the window.
 """
 from __future__ import annotations
 
+import bisect
 from dataclasses import dataclass, field
 
 from .ir import Program
@@ -254,6 +255,11 @@ class _Window:
         self.reexec = {}         # j -> supplies (per operand register, uses() order)
         self.events = []         # establishment order
         ins = prog.instrs
+        # sorted def positions of every register inside the window [p, c)
+        self.defs = {}
+        for k in range(p, c):
+            if ins[k].defreg is not None:
+                self.defs.setdefault(ins[k].defreg, []).append(k)
         for r in prog.all_regs():
             self.valid[(r, self.rd(r, c))] = ("C",)
         for m in sorted(backups):
@@ -265,17 +271,19 @@ class _Window:
 
     # rd(r, t): last def of r in [p, t), else PRE
     def rd(self, r, t):
-        for k in range(t - 1, self.p - 1, -1):
-            if self.prog.instrs[k].defreg == r:
-                return k
-        return PRE
+        d = self.defs.get(r)
+        if not d:
+            return PRE
+        i = bisect.bisect_left(d, t)
+        return d[i - 1] if i > 0 else PRE
 
     # nd(r, t): first def of r in [t, c), else None
     def nd(self, r, t):
-        for k in range(t, self.c):
-            if self.prog.instrs[k].defreg == r:
-                return k
-        return None
+        d = self.defs.get(r)
+        if not d:
+            return None
+        i = bisect.bisect_left(d, t)
+        return d[i] if i < len(d) else None
 
     def is_current(self, v):
         r, d = v

@@ -54,10 +54,16 @@ struct ctxb_program {
   CodegenInfo cg;
   std::string src, log;
   std::vector<char> cubin;
-  uint32_t num_regs = 0;
+  uint32_t num_regs = 0, regs_resume = 0;
   double t_an = 0, t_cg = 0, t_cc = 0;
   std::mutex mu;
   std::map<CUcontext, Mod> mods;
+  struct Res {
+    CUdeviceptr flag = 0, stamps = 0, forced = 0;
+    uint32_t n_warps = 0;
+    CUevent ev0 = nullptr, ev1 = nullptr;
+  };
+  std::vector<Res> pool;   // per-run device resources, reused (flag is always left at 0)
   uint32_t full_ir_words128() const {  // 128-B rows occupied by the FULL_IR layout
     return (uint32_t)prog.nv + ((uint32_t)prog.ns * 4 + 127) / 128;
   }
@@ -91,12 +97,11 @@ struct ctxb_run {
   int state = RUN_RUNNING;
   std::vector<uint32_t> hdr_prev, hdr;  // host header snapshots (launch e-1, e)
   bool resumed_launch = false;
+  CUevent ev0 = nullptr, ev1 = nullptr;   // recorded around each launch on the run's stream
   ~ctxb_run() {
-    Driver& d = driver();
-    if (d.ok) {
-      if (flag) d.cuMemFree(flag);
-      if (stamps) d.cuMemFree(stamps);
-      if (forced) d.cuMemFree(forced);
+    if (flag && prog) {   // return the resources to the program's pool
+      std::lock_guard<std::mutex> g(prog->mu);
+      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1});
     }
   }
 };
@@ -139,7 +144,7 @@ int ensure_module(ctxb_program* p, CUcontext c, Mod* out) {
   return CTXB_OK;
 }
 
-int compile(ctxb_program* p) {
+int nvrtc_compile(ctxb_program* p, uint32_t* regs_run, uint32_t* regs_resume) {
   Nvrtc& n = nvrtc();
   if (!n.ok) return fail(CTXB_E_NVRTC, n.err);
   void* prog = nullptr;
@@ -162,13 +167,44 @@ int compile(ctxb_program* p) {
   p->cubin.resize(cs);
   n.GetCUBIN(prog, p->cubin.data());
   n.DestroyProgram(&prog);
-  // ptxas -v: "Compiling entry function 'ctxb_run'" ... "Used N registers"
-  size_t at = log.find("'ctxb_run'");
-  if (at != std::string::npos) {
+  // ptxas -v: "Compiling entry function 'NAME'" ... "Used N registers"
+  auto regs_of = [&](const char* fn) -> uint32_t {
+    size_t at = log.find(std::string("'") + fn + "'");
+    if (at == std::string::npos) return 0;
     std::smatch m;
     std::string tail = log.substr(at);
-    if (std::regex_search(tail, m, std::regex("Used ([0-9]+) registers"))) p->num_regs = (uint32_t)std::stoul(m[1]);
+    if (std::regex_search(tail, m, std::regex("Used ([0-9]+) registers"))) return (uint32_t)std::stoul(m[1]);
+    return 0;
+  };
+  *regs_run = regs_of("ctxb_run");
+  *regs_resume = regs_of("ctxb_resume");
+  return CTXB_OK;
+}
+
+// Resident blocks per SM allowed by the register file (64 K 32-bit registers,
+// per-warp allocation in units of 256 registers, at most 64 warps / 32 blocks).
+uint32_t blocks_by_regs(uint32_t regs, uint32_t block) {
+  if (regs == 0) return 32;
+  uint32_t warps = (block + 31) / 32;
+  uint32_t per_warp = ((regs * 32 + 255) / 256) * 256;
+  uint32_t b = 65536u / (per_warp * warps);
+  return std::min<uint32_t>(std::min<uint32_t>(b, 64u / warps), 32u);
+}
+
+int compile(ctxb_program* p) {
+  uint32_t rr = 0, rs = 0;
+  int rc = nvrtc_compile(p, &rr, &rs);
+  if (rc) return rc;
+  uint32_t bw = blocks_by_regs(rr, p->prog.block), bs = blocks_by_regs(rs, p->prog.block);
+  if (bs < bw && bw > 0) {
+    // ask ptxas for the normal kernel's occupancy (__launch_bounds__ min blocks)
+    p->cg.resume_maxnreg = bw;
+    p->src = generate_cuda(p->prog, p->an, p->opt, &p->cg);
+    rc = nvrtc_compile(p, &rr, &rs);
+    if (rc) return rc;
   }
+  p->num_regs = rr;
+  p->regs_resume = rs;
   return CTXB_OK;
 }
 
@@ -210,8 +246,10 @@ int launch(ctxb_run* r, bool resume) {
   pack_params(r, r->prog, blob);
   void* args[] = {blob.data()};
   Driver& d = driver();
+  CU(d.cuEventRecord(r->ev0, r->stream));
   CU(d.cuLaunchKernel(resume ? r->mod.resume : r->mod.run, r->grid, 1, 1, (unsigned)r->prog->prog.block, 1, 1, 0,
                       r->stream, args, nullptr));
+  CU(d.cuEventRecord(r->ev1, r->stream));
   r->state = RUN_RUNNING;
   r->resumed_launch = resume;
   return CTXB_OK;
@@ -255,10 +293,12 @@ const char* ctxb_version(void) { return "ctxb 0.1 (sm_100a, CTXB-R1)"; }
 int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb_program** out) {
   if (!ir_text || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   *out = nullptr;
-  ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0};
-  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 7) return fail(CTXB_E_INVALID_ARG, "bad options");
+  ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0};
+  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 7 || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
+    return fail(CTXB_E_INVALID_ARG, "bad options");
   std::unique_ptr<ctxb_program> p(new ctxb_program);
-  p->opt = Options{o.flags, o.mode, o.poll_policy, o.poll_every ? o.poll_every : 8, o.debug};
+  p->opt = Options{o.flags, o.mode, o.poll_policy, o.poll_every ? o.poll_every : 8, o.debug,
+                   o.flag_depth ? o.flag_depth : 1, o.min_blocks_per_sm};
   try {
     double t0 = now_ms();
     p->prog = parse_ir(std::string(ir_text, len));
@@ -286,8 +326,16 @@ int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb
 int ctxb_program_destroy(ctxb_program* p) {
   if (!p) return fail(CTXB_E_INVALID_ARG, "NULL program");
   Driver& d = driver();
-  if (d.ok)
+  if (d.ok) {
     for (auto& [c, m] : p->mods) d.cuModuleUnload(m.mod);
+    for (auto& r : p->pool) {
+      d.cuMemFree(r.flag);
+      d.cuMemFree(r.stamps);
+      d.cuMemFree(r.forced);
+      d.cuEventDestroy(r.ev0);
+      d.cuEventDestroy(r.ev1);
+    }
+  }
   delete p;
   return CTXB_OK;
 }
@@ -306,6 +354,8 @@ int ctxb_program_info(const ctxb_program* p, ctxb_program_info_t* o) {
   o->full_ir_bytes_per_warp = p->an.full_ir_bytes;
   o->num_regs = p->num_regs;
   o->compiled = p->cubin.empty() ? 0 : 1;
+  o->num_regs_resume = p->regs_resume;
+  o->resume_maxnreg = p->cg.resume_maxnreg;
   o->analyze_ms = p->t_an;
   o->codegen_ms = p->t_cg;
   o->compile_ms = p->t_cc;
@@ -352,6 +402,26 @@ int ctxb_generated_source(const ctxb_program* p, char* buf, size_t cap, size_t* 
   return copy_out(p->src, buf, cap, len);
 }
 
+int ctxb_occupancy(ctxb_program* p, uint32_t* bps, uint32_t* nsm) {
+  if (!p || !bps || !nsm) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  CUcontext c;
+  int rc = ensure_ctx(&c);
+  if (rc) return rc;
+  Mod m;
+  rc = ensure_module(p, c, &m);
+  if (rc) return rc;
+  Driver& d = driver();
+  int a = 0, b = 0, n = 0;
+  CU(d.cuOccupancyMaxActiveBlocksPerMultiprocessor(&a, m.run, p->prog.block, 0));
+  CU(d.cuOccupancyMaxActiveBlocksPerMultiprocessor(&b, m.resume, p->prog.block, 0));
+  CUdevice dev;
+  CU(d.cuCtxGetDevice(&dev));
+  CU(d.cuDeviceGetAttribute(&n, CU_DEVICE_ATTRIBUTE_MULTIPROCESSOR_COUNT, dev));
+  *bps = (uint32_t)std::min(a, b);
+  *nsm = (uint32_t)n;
+  return CTXB_OK;
+}
+
 int ctxb_context_capacity(const ctxb_program* p, uint32_t grid, uint64_t* bytes) {
   if (!p || !bytes || grid == 0) return fail(CTXB_E_INVALID_ARG, "bad argument");
   if (p->opt.mode == CTXB_MODE_FULL_HW && p->num_regs == 0)
@@ -393,12 +463,34 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
   r->pay_off = (((uint64_t)r->n_warps * 16 + 255) / 256) * 256;
   r->stride = p->stride();
   r->stream = (CUstream)stream;
-  CU(d.cuMemAlloc(&r->flag, 256));
-  CU(d.cuMemAlloc(&r->stamps, (size_t)r->n_warps * 32));
-  CU(d.cuMemAlloc(&r->forced, (size_t)r->n_warps * 4));
-  CU(d.cuMemsetD32Async(r->flag, 0, 64, r->stream));
-  CU(d.cuMemsetD32Async(r->stamps, 0, (size_t)r->n_warps * 8, r->stream));
-  CU(d.cuMemsetD32Async(r->cbuf, 0, (size_t)r->n_warps * 4, r->stream));   // headers
+  {
+    std::lock_guard<std::mutex> g(p->mu);
+    for (size_t i = 0; i < p->pool.size(); i++)
+      if (p->pool[i].n_warps == r->n_warps) {
+        r->flag = p->pool[i].flag;
+        r->stamps = p->pool[i].stamps;
+        r->forced = p->pool[i].forced;
+        r->ev0 = p->pool[i].ev0;
+        r->ev1 = p->pool[i].ev1;
+        p->pool.erase(p->pool.begin() + (long)i);
+        break;
+      }
+  }
+  if (!r->flag) {
+    CUdeviceptr f = 0, s = 0, t = 0;
+    CU(d.cuMemAlloc(&f, 256));
+    CU(d.cuMemAlloc(&s, (size_t)r->n_warps * 32));
+    CU(d.cuMemAlloc(&t, (size_t)r->n_warps * 4));
+    r->flag = f;
+    r->stamps = s;
+    r->forced = t;
+    CU(d.cuEventCreate(&r->ev0, CU_EVENT_DEFAULT));
+    CU(d.cuEventCreate(&r->ev1, CU_EVENT_DEFAULT));
+    std::vector<uint32_t> z(64, 0);
+    CU(d.cuMemcpyHtoD(r->flag, z.data(), 256));   // the flag is 0 whenever a run does not hold it raised
+  }
+  // No header memset: every warp of launch 0 writes its header (DONE or
+  // PREEMPTED with epoch 1) before the launch completes.
   rc = upload_forced(r.get(), forced_targets);
   if (rc) return rc;
   r->epoch = 1;
@@ -467,6 +559,15 @@ int ctxb_wait(ctxb_run* r, int* finished) {
     if (rc) return rc;
   }
   if (finished) *finished = r->state == RUN_DONE ? 1 : 0;
+  return CTXB_OK;
+}
+
+int ctxb_launch_ms(const ctxb_run* r, float* ms) {
+  if (!r || !ms) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  if (r->state == RUN_RUNNING) return fail(CTXB_E_STATE, "launch still running: call ctxb_wait/ctxb_preempt first");
+  Driver& d = driver();
+  CU(d.cuEventSynchronize(r->ev1));
+  CU(d.cuEventElapsedTime(ms, r->ev0, r->ev1));
   return CTXB_OK;
 }
 

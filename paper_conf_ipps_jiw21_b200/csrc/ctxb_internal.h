@@ -137,7 +137,7 @@ struct Plan {
 };
 
 struct Options {
-  uint32_t flags = 7, mode = 0, policy = 0, every = 8, debug = 0;
+  uint32_t flags = 7, mode = 0, policy = 0, every = 8, debug = 0, flag_depth = 1, min_blocks = 0;
 };
 
 struct Analysis {
@@ -157,6 +157,7 @@ std::string plan_text(const Program& prog, const Plan& pl);
 struct CodegenInfo {
   uint32_t stride = 0;            // payload slot bytes per warp (multiple of 128)
   uint32_t max_payload = 0;
+  uint32_t resume_maxnreg = 0;    // in: register cap of the resume kernel (0 = none)
 };
 std::string generate_cuda(const Program& prog, const Analysis& an, const Options& opt,
                           CodegenInfo* info);

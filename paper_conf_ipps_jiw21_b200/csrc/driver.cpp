@@ -46,7 +46,11 @@ Driver& driver() {
               sym(h, "cuMemcpyHtoDAsync_v2", &d.cuMemcpyHtoDAsync, &e) &&
               sym(h, "cuMemsetD32Async", &d.cuMemsetD32Async, &e) && sym(h, "cuMemsetD8Async", &d.cuMemsetD8Async, &e) &&
               sym(h, "cuStreamSynchronize", &d.cuStreamSynchronize, &e) &&
-              sym(h, "cuGetErrorString", &d.cuGetErrorString, &e);
+              sym(h, "cuGetErrorString", &d.cuGetErrorString, &e) &&
+              sym(h, "cuEventCreate", &d.cuEventCreate, &e) && sym(h, "cuEventRecord", &d.cuEventRecord, &e) &&
+              sym(h, "cuEventSynchronize", &d.cuEventSynchronize, &e) &&
+              sym(h, "cuEventElapsedTime", &d.cuEventElapsedTime, &e) &&
+              sym(h, "cuEventDestroy_v2", &d.cuEventDestroy, &e);
     if (ok && !sym(h, "cuStreamWriteValue32_v2", &d.cuStreamWriteValue32, &e))
       ok = sym(h, "cuStreamWriteValue32", &d.cuStreamWriteValue32, &e);
     if (!ok) return;

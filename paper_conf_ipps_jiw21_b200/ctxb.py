@@ -34,8 +34,8 @@ NEVER = 0xFFFFFFFF
 EXPORTED_SYMBOLS = [
     "ctxb_last_error", "ctxb_version", "ctxb_analyze", "ctxb_program_destroy", "ctxb_program_info",
     "ctxb_num_sites", "ctxb_site_info", "ctxb_backups", "ctxb_site_plan_text", "ctxb_generated_source",
-    "ctxb_context_capacity", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait",
-    "ctxb_resume_stats_get", "ctxb_context_bytes", "ctxb_read_headers", "ctxb_read_stamps",
+    "ctxb_occupancy", "ctxb_context_capacity", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait",
+    "ctxb_launch_ms", "ctxb_resume_stats_get", "ctxb_context_bytes", "ctxb_read_headers", "ctxb_read_stamps",
     "ctxb_run_destroy",
 ]
 
@@ -48,7 +48,8 @@ class CtxbError(RuntimeError):
 
 class _Opts(C.Structure):
     _fields_ = [("flags", C.c_uint32), ("mode", C.c_uint32), ("poll_policy", C.c_uint32),
-                ("poll_every", C.c_uint32), ("debug", C.c_uint32)]
+                ("poll_every", C.c_uint32), ("debug", C.c_uint32), ("flag_depth", C.c_uint32),
+                ("min_blocks_per_sm", C.c_uint32)]
 
 
 class _SiteInfo(C.Structure):
@@ -59,7 +60,7 @@ class _SiteInfo(C.Structure):
 class _ProgInfo(C.Structure):
     _fields_ = [(n, C.c_uint32) for n in ("n_instrs", "nv", "ns", "block", "n_buffers", "n_uniforms", "n_sites",
                                           "n_backups", "max_payload_bytes_per_warp", "full_ir_bytes_per_warp",
-                                          "num_regs", "compiled")] + \
+                                          "num_regs", "compiled", "num_regs_resume", "resume_maxnreg")] + \
                [("analyze_ms", C.c_double), ("codegen_ms", C.c_double), ("compile_ms", C.c_double)]
 
 
@@ -91,11 +92,13 @@ def _load():
         "ctxb_site_plan_text": (I, [P, U32, I, C.c_char_p, SZ, C.POINTER(SZ)]),
         "ctxb_generated_source": (I, [P, C.c_char_p, SZ, C.POINTER(SZ)]),
         "ctxb_context_capacity": (I, [P, U32, C.POINTER(U64)]),
+        "ctxb_occupancy": (I, [P, C.POINTER(U32), C.POINTER(U32)]),
         "ctxb_launch": (I, [P, U32, C.POINTER(P), C.POINTER(U32), P, U64, P, C.POINTER(U32), C.POINTER(P)]),
         "ctxb_preempt": (I, [P, P, C.POINTER(_PreStats)]),
         "ctxb_resume": (I, [P, P, C.POINTER(U32)]),
         "ctxb_wait": (I, [P, C.POINTER(I)]),
         "ctxb_resume_stats_get": (I, [P, C.POINTER(_ResStats)]),
+        "ctxb_launch_ms": (I, [P, C.POINTER(C.c_float)]),
         "ctxb_context_bytes": (I, [P, C.POINTER(U64), C.POINTER(U64), C.POINTER(U32)]),
         "ctxb_read_headers": (I, [P, C.POINTER(U32), U64]),
         "ctxb_read_stamps": (I, [P, C.POINTER(U64), U64]),
@@ -142,8 +145,8 @@ def _u32arr(vals):
 # --- the C-ABI names ----------------------------------------------------------
 
 def ctxb_analyze(ir_text: str, flags=ALL, mode=MODE_CTXBACK, poll_policy=POLL_EVERY_INSTR, poll_every=8,
-                 debug=0) -> "Program":
-    return Program(ir_text, flags, mode, poll_policy, poll_every, debug)
+                 debug=0, flag_depth=1, min_blocks_per_sm=0) -> "Program":
+    return Program(ir_text, flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm)
 
 
 def ctxb_launch(prog, grid, buffers, uniforms, ctx, stream=None, forced=None) -> "Run":
@@ -170,9 +173,9 @@ class Program:
     """An analysed + compiled IR kernel (ctxb_analyze)."""
 
     def __init__(self, ir_text, flags=ALL, mode=MODE_CTXBACK, poll_policy=POLL_EVERY_INSTR, poll_every=8,
-                 debug=0):
+                 debug=0, flag_depth=1, min_blocks_per_sm=0):
         self._h = C.c_void_p()
-        o = _Opts(flags, mode, poll_policy, poll_every, debug)
+        o = _Opts(flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm)
         b = ir_text.encode()
         _chk(lib.ctxb_analyze(b, len(b), C.byref(o), C.byref(self._h)))
         self.debug = debug
@@ -223,6 +226,12 @@ class Program:
     def source(self):
         return self._text(lib.ctxb_generated_source)
 
+    def occupancy(self):
+        """(resident blocks per SM, number of SMs) -> persistent grid = product."""
+        a, n = C.c_uint32(), C.c_uint32()
+        _chk(lib.ctxb_occupancy(self._h, C.byref(a), C.byref(n)))
+        return a.value, n.value
+
     def context_capacity(self, grid):
         b = C.c_uint64()
         _chk(lib.ctxb_context_capacity(self._h, grid, C.byref(b)))
@@ -271,6 +280,12 @@ class Run:
         fin = C.c_int()
         _chk(lib.ctxb_wait(self._h, C.byref(fin)))
         return bool(fin.value)
+
+    def launch_ms(self):
+        """Device duration of the last launch (library-recorded CUDA events)."""
+        f = C.c_float()
+        _chk(lib.ctxb_launch_ms(self._h, C.byref(f)))
+        return f.value
 
     def resume_stats(self):
         s = _ResStats()

@@ -1,0 +1,139 @@
+"""GPU parity on the BASELINE.json configs beyond C1 (C2 tiled SGEMM), and the
+bulk save/restore microbench's correctness.
+
+* C2 at a small size: the generated kernel's C equals the oracle interpreter's
+  bit for bit, uninterrupted and under forced random per-warp preemption
+  (nested, poisoned), with per-warp context bytes equal to the oracle's;
+* C2 at the full BASELINE size (4096^3, 148 SMs x occupancy persistent grid):
+  sampled C elements equal the oracle's correctly rounded f32 fma chain in the
+  IR's k order; preemption by the flag at random times + resume gives C
+  bit-exact with the uninterrupted run; every preempted warp's header bytes
+  equal the oracle plan's bytes for the site it reports.
+"""
+import numpy as np
+import pytest
+
+from oracle import analysis as A
+from oracle import fp32, interp, ir
+from workloads import configs
+
+from gpu_helpers import from_dev, gpu_run, header_records, oracle_records, to_dev
+
+pytestmark = pytest.mark.gpu
+
+
+def _cb():
+    import paper_conf_ipps_jiw21_b200 as cb
+    return cb
+
+
+@pytest.mark.parametrize("size,grid,nsched,polls", [((128, 128, 64), 1, 3, "iter"), ((128, 128, 32), 1, 3, "half"),
+                                                    ((256, 256, 32), 4, 1, "iter")])
+def test_c2_small_forced(size, grid, nsched, polls):
+    cb = _cb()
+    M, N, K = size
+    cfg = configs.c2(M, N, K, polls=polls)
+    op = ir.parse(cfg["ir"])
+    an = A.analyze(op, policy="EXPLICIT")
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_FORCED | cb.DEBUG_POISON,
+                      min_blocks_per_sm=cfg["min_blocks"])
+    for k, c in enumerate(an.sites):
+        assert prog.plan_text(k) == A.plan_text(op, an.plans[c])
+    names = list(op.buffers)
+    ref, _ = interp.run(an, grid, cfg["buffers"])
+    g0, _h, _ = gpu_run(prog, names, grid, cfg["buffers"], {})
+    assert np.array_equal(g0["C"], ref["C"])
+    per_iter = {"iter": 1, "step": 4, "half": 8}[polls]
+    visits = (K // 4) * per_iter * (M * N // (128 * 128) // grid)
+    r = np.random.default_rng(5)
+    nw = grid * 8
+    for _ in range(nsched):
+        sched = [r.integers(0, visits, nw).astype(np.uint32), r.integers(0, 40, nw).astype(np.uint32)]
+        out, rec = interp.run(an, grid, cfg["buffers"], schedule=sched)
+        assert np.array_equal(out["C"], ref["C"])
+        g, hdrs, _ = gpu_run(prog, names, grid, cfg["buffers"], {}, schedule=sched)
+        assert np.array_equal(g["C"], ref["C"])
+        assert header_records(hdrs)[:len(oracle_records(rec, an))] == oracle_records(rec, an)
+
+
+def test_c2_full_size_flag_preemption():
+    import time
+    import torch
+    cb = _cb()
+    cfg = configs.c2()
+    M, N, K = cfg["M"], cfg["N"], cfg["K"]
+    op = ir.parse(cfg["ir"])
+    an = A.analyze(op, policy="EXPLICIT")
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=cfg["min_blocks"])
+    for k, c in enumerate(an.sites):
+        assert prog.plan_text(k) == A.plan_text(op, an.plans[c])
+    bps, nsm = prog.occupancy()
+    assert bps == 2
+    grid = bps * nsm
+    dA, dB = to_dev(cfg["buffers"]["A"]), to_dev(cfg["buffers"]["B"])
+    dC = torch.zeros(M * N, dtype=torch.int32, device="cuda")
+    ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    s = torch.cuda.Stream()
+    ctrl = torch.cuda.Stream()
+    t0 = time.time()
+    run = prog.launch(grid, [dA, dB, dC], [], ctx, s)
+    assert run.wait()
+    t_unint = time.time() - t0
+    ref = dC.clone()
+    # sampled elements vs the oracle's f32 fma chain in the IR's k order
+    rng = np.random.default_rng(17)
+    rows = rng.integers(0, M, 256)
+    cols = rng.integers(0, N, 256)
+    A_ = cfg["buffers"]["A"]
+    B_ = cfg["buffers"]["B"]
+    acc = np.zeros(256, dtype=np.uint32)
+    for k in range(K):
+        acc = fp32.ffma(A_[rows * K + k], B_[k * N + cols], acc)
+    got = from_dev(ref)[rows * N + cols]
+    assert np.array_equal(got, acc)
+    site_bytes = {k: an.plans[c].payload_bytes for k, c in enumerate(an.sites)}
+    live_bytes = {k: an.live[c].payload_bytes for k, c in enumerate(an.sites)}
+    for trial in range(3):
+        dC.zero_()
+        torch.cuda.synchronize()
+        run = prog.launch(grid, [dA, dB, dC], [], ctx, s)
+        time.sleep(t_unint * (0.1 + 0.3 * trial))
+        st = run.preempt(ctrl)
+        if st["warps_preempted"]:
+            h = run.headers()
+            for w in range(h.shape[0]):
+                if h[w, 2] == 1 and h[w, 3] == 1:
+                    k, live = int(h[w, 0]) & 0x7FFFFFFF, bool(h[w, 0] >> 31)
+                    assert int(h[w, 1]) == (live_bytes[k] if live else site_bytes[k])
+            assert st["payload_bytes"] == run.context_bytes()[0]
+            run.resume(s)
+            assert run.wait()
+        torch.cuda.synchronize()
+        assert torch.equal(dC, ref), f"trial {trial}: C after preempt/resume differs"
+
+
+def test_bulk_save_restore_roundtrip():
+    import torch
+    cb = _cb()
+    prog = cb.Program(configs.bulk_ir(64), poll_policy=cb.POLL_EXPLICIT, mode=cb.MODE_LIVE,
+                      debug=cb.DEBUG_FORCED)
+    grid = 2048
+    nw = grid * 8
+    out = torch.zeros(256, dtype=torch.int32, device="cuda")
+    ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    run = prog.launch(grid, [out], [], ctx, forced=np.zeros(nw, np.uint32))
+    assert not run.wait()
+    h = run.headers()
+    assert (h[:, 2] == 1).all() and (h[:, 1] == 64 * 128).all()
+    # payload of warp w: group g lane l holds values 4g..4g+3 of thread 32*(w%8)+l
+    pay_off = ((nw * 16 + 255) // 256) * 256
+    raw = ctx[pay_off:pay_off + 8 * 8192].cpu().numpy().view(np.uint32).reshape(8, 16, 32, 4)
+    tid = (np.arange(8)[:, None] * 32 + np.arange(32)[None, :]).astype(np.uint32)
+    for g in range(16):
+        for q in range(4):
+            i = 4 * g + q
+            want = tid ^ np.uint32(((i + 1) * 0x9E3779B9) & 0xFFFFFFFF)
+            assert np.array_equal(raw[:, g, :, q], want)
+    run.resume(forced=np.full(nw, cb.NEVER, np.uint32))
+    assert run.wait()
+    assert int(out.abs().sum()) == 0
