@@ -275,7 +275,7 @@ def peaks():
 def ncu_traffic():
     """Per-launch DRAM traffic of the bulk save / restore kernels from the
     committed ncu --set full capture (profiles/), if present."""
-    p = os.path.join(ROOT, "profiles", "ncu_bulk_traffic.json")
+    p = os.path.join(ROOT, "profiles", "ncu_bulk_traffic.json")   # written from round-1 ncu capture
     if os.path.exists(p):
         try:
             return json.load(open(p))
