@@ -78,3 +78,27 @@ def oracle_records(records, an):
         out.setdefault(r["launch"], {})[r["warp"]] = (idx[c], live, r["bytes"])
     n = max(out) + 1 if out else 0
     return [out.get(k, {}) for k in range(n)]
+
+
+def flag_run(prog, grid, dev_buffers, uniforms, ctx, delay_s, stream, ctrl):
+    """Launch, raise the preemption flag after `delay_s` (host clock), resume
+    until done.  Returns the preempt stats (or None if the run finished
+    first) and the header array of the preempted launch."""
+    import time
+    run = prog.launch(grid, dev_buffers, uniforms, ctx, stream)
+    t0 = time.perf_counter()
+    while time.perf_counter() < t0 + delay_s:
+        pass
+    st = run.preempt(ctrl)
+    hdr = run.headers().copy()
+    if st["warps_preempted"]:
+        run.resume(stream)
+        assert run.wait()
+    return st, hdr, run
+
+
+def check_headers_vs_plans(hdr, epoch, site_bytes, live_bytes):
+    for w in range(hdr.shape[0]):
+        if hdr[w, 2] == 1 and hdr[w, 3] == epoch:
+            k, live = int(hdr[w, 0]) & 0x7FFFFFFF, bool(hdr[w, 0] >> 31)
+            assert int(hdr[w, 1]) == (live_bytes[k] if live else site_bytes[k]), (w, hdr[w])

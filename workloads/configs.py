@@ -199,3 +199,231 @@ def bulk_ir(nvals=64, block=256):
     e(f"  @v{n} stg out[%tid], v0")
     e("  exit")
     return "\n".join(L) + "\n"
+
+
+# configs[2]: "2D 5-point stencil IR kernel with loop-carried induction
+# registers (exercises instruction reverting)".
+def c3_ir(W=8192, H=8192, strip=64, polls="both"):
+    """y = 0.5*x + 0.125*(N + S + W + E) on interior points (f32, IR order:
+    ((N + S) + W) + E, then * 0.125, then 0.5*x + that).  Thread per column,
+    256 columns x `strip` rows per work item; persistent grid, item = ctaid +
+    i*nctaid.  Per row: five loads around idx, the sum, then the loop-carried
+    induction registers advance (idx += W, row += 1: reversible IADDs) and the
+    finished value is written behind at idx - W.  Polls: in the middle of the
+    sum, and after the advance (there CTXBack reverts idx += W at resume and
+    re-executes the loads and the sum instead of saving the result)."""
+    assert W % 256 == 0 and H % strip == 0
+    ncb = W // 256
+    items = ncb * (H // strip)
+    L = [".kernel c3_stencil", ".buffer ro X", ".buffer wo Y", ".vregs 12", ".sregs 8", ".block 256"]
+    e = L.append
+    e("init:")
+    e("  mov s6, %ctaid")                               # work item
+    e("item:")
+    e(f"  setp.lt.u s7, s6, {items}")
+    e("  brz s7, done")
+    e("setup:")
+    e(f"  and s0, s6, {ncb - 1}")                       # column block
+    shift = ncb.bit_length() - 1
+    e(f"  shr s1, s6, {shift}")                         # strip index
+    e("  shl s2, s0, 8")
+    e("  iadd v0, s2, %tid")                            # col
+    e(f"  imul s3, s1, {strip}")                        # row
+    e("  setp.gt.u v1, v0, 0")
+    e(f"  setp.lt.u v2, v0, {W - 1}")
+    e("  and v1, v1, v2")                               # interior column
+    e(f"  imad v3, s3, {W}, v0")                        # idx of (row, col)
+    e(f"  mov s5, {strip}")
+    e("rows:")
+    e("  setp.gt.u s4, s3, 0")                          # row > 0
+    e(f"  setp.lt.u s2, s3, {H - 1}")                   # row < H-1
+    e("  and s4, s4, s2")                               # interior row
+    e("  and v11, v1, s4")                              # interior point
+    e(f"  isub v4, v3, {W}")
+    e("  @v11 ldg v5, X[v4]")                           # north
+    e(f"  iadd v4, v3, {W}")
+    e("  @v11 ldg v6, X[v4]")                           # south
+    e("  isub v4, v3, 1")
+    e("  @v11 ldg v7, X[v4]")                           # west
+    e("  iadd v4, v3, 1")
+    e("  @v11 ldg v8, X[v4]")                           # east
+    e("  ldg v9, X[v3]")                                # centre
+    e("  fadd v10, v5, v6")
+    e("  fadd v10, v10, v7")
+    if polls in ("both", "mid"):
+        e("  poll")
+    e("  fadd v10, v10, v8")
+    e("  fmul v10, v10, 0f3E000000")                    # * 0.125
+    e("  fmul v9, v9, 0f3F000000")                      # 0.5 * x
+    e("  fadd v10, v9, v10")
+    e(f"  iadd v3, v3, {W}")                            # idx += W   (reversible)
+    e("  iadd s3, s3, 1")                               # row += 1   (reversible)
+    if polls in ("both", "end"):
+        e("  poll")
+    e(f"  isub v4, v3, {W}")                            # write behind at the old idx
+    e("  @v11 stg Y[v4], v10")
+    e("  isub s5, s5, 1")
+    e("  brnz s5, rows")
+    e("next:")
+    e("  iadd s6, s6, %nctaid")
+    e("  bra item")
+    e("done:")
+    e("  exit")
+    return "\n".join(L) + "\n"
+
+
+def c3(W=8192, H=8192, strip=64, polls="both"):
+    r = np.random.default_rng(21)
+    bufs = {"X": f32_bits(r.uniform(0.0, 1.0, W * H).astype(np.float32)),
+            "Y": np.zeros(W * H, dtype=np.uint32)}
+    return dict(name="C3", ir=c3_ir(W, H, strip, polls), grid=None, buffers=bufs, uniforms={},
+                policy="EXPLICIT", W=W, H=H, strip=strip, min_blocks=0)
+
+
+def c3_numpy_reference(x_bits, W, H):
+    """Textbook f32 5-point stencil in the IR's operation order (test pin)."""
+    x = x_bits.view(np.float32).reshape(H, W)
+    y = np.zeros((H, W), dtype=np.float32)
+    n, s = x[:-2, 1:-1], x[2:, 1:-1]
+    w, e = x[1:-1, :-2], x[1:-1, 2:]
+    acc = ((n + s) + w) + e
+    acc = acc * np.float32(0.125)
+    y[1:-1, 1:-1] = x[1:-1, 1:-1] * np.float32(0.5) + acc
+    return y.reshape(-1).view(np.uint32)
+
+
+# configs[3]: "histogram + BFS-frontier IR kernels with scalar-operand-limited
+# re-execution (exercises on-chip scalar backup)".
+def c4a_ir(nkeys=1 << 28, per_lane=8):
+    """256-bin histogram of u32 keys (bin = key >> 24) with global atomics.
+    Warp-cooperative chunk loop: a warp handles chunks of 32*per_lane keys;
+    the chunk base is a scalar loaded from `starts` (an irreversible uniform
+    load that overwrites the base the chunk's key loads were addressed from --
+    the OSRB case).  One poll per chunk, after the next base is
+    loaded and before the atomics."""
+    chunk = 32 * per_lane
+    assert nkeys % chunk == 0
+    nch = nkeys // chunk
+    L = [".kernel c4a_hist", ".buffer ro keys", ".buffer ro starts", ".buffer rw hist",
+         f".vregs {1 + 2 * per_lane}", ".sregs 6", ".block 256"]
+    e = L.append
+    e("init:")
+    e("  imad s0, %ctaid, %nwarps, %warpid")          # chunk index = global warp id
+    e("  imul s1, %nctaid, %nwarps")                  # total warps
+    e(f"  setp.lt.u s2, s0, {nch}")
+    e("  brz s2, done")
+    e("first:")
+    e("  ldg s3, starts[s0]")                         # base of the first chunk
+    e("loop:")
+    e("  iadd v0, s3, %laneid")
+    for j in range(per_lane):
+        e(f"  ldg v{1 + j}, keys[v0]")
+        if j + 1 < per_lane:
+            e("  iadd v0, v0, 32")
+    for j in range(per_lane):
+        e(f"  shr v{1 + per_lane + j}, v{1 + j}, 24")
+    e("  iadd s0, s0, s1")                            # next chunk (reversible)
+    e(f"  setp.lt.u s2, s0, {nch}")
+    e(f"  umin s4, s0, {nch - 1}")
+    e("  ldg s3, starts[s4]")                         # next base: irreversible scalar overwrite
+    e("  poll")
+    for j in range(per_lane):
+        e(f"  atom.add _, hist[v{1 + per_lane + j}], 1")
+    e("  brnz s2, loop")
+    e("done:")
+    e("  exit")
+    return "\n".join(L) + "\n"
+
+
+def c4a(nkeys=1 << 28, skewed=False, per_lane=8):
+    chunk = 32 * per_lane
+    if skewed:
+        r = np.random.default_rng(32)
+        u = r.random(nkeys, dtype=np.float64)
+        keys = np.floor((u ** 4) * 4294967296.0).astype(np.uint64).clip(0, 0xFFFFFFFF).astype(np.uint32)
+    else:
+        r = np.random.default_rng(31)
+        keys = r.integers(0, 1 << 32, nkeys, dtype=np.uint64).astype(np.uint32)
+    starts = (np.arange(nkeys // chunk, dtype=np.uint64) * chunk).astype(np.uint32)
+    bufs = {"keys": keys, "starts": starts, "hist": np.zeros(256, dtype=np.uint32)}
+    return dict(name="C4a", ir=c4a_ir(nkeys, per_lane), grid=None, buffers=bufs, uniforms={},
+                policy="EXPLICIT", nkeys=nkeys, min_blocks=0)
+
+
+def c4b_ir():
+    """One level of a level-synchronous top-down BFS: warp per frontier vertex
+    (scalar v, edge range [beg, end) from irreversible uniform loads), lanes
+    over its edges; dist[u] claimed with atomicCAS(INF -> level+1) and newly
+    discovered vertices pushed with atomicAdd on the next-frontier counter.
+    Polls: after the vertex's loads and before each edge chunk's atomics."""
+    L = [".kernel c4b_bfs", ".buffer ro rowptr", ".buffer ro colidx", ".buffer ro front",
+         ".buffer rw dist", ".buffer rw nextf", ".buffer rw nextcnt", ".uniform nf", ".uniform lvl1",
+         ".vregs 6", ".sregs 8", ".block 256"]
+    e = L.append
+    e("init:")
+    e("  imad s0, %ctaid, %nwarps, %warpid")          # frontier index = global warp id
+    e("  imul s1, %nctaid, %nwarps")
+    e("vloop:")
+    e("  setp.lt.u s2, s0, %nf")
+    e("  brz s2, done")
+    e("vbody:")
+    e("  ldg s3, front[s0]")                          # v          (irreversible)
+    e("  ldg s4, rowptr[s3]")                         # beg        (irreversible)
+    e("  iadd s5, s3, 1")
+    e("  ldg s5, rowptr[s5]")                         # end        (irreversible, reads old s5)
+    e("  mov s6, s4")                                 # e = beg
+    e("  poll")
+    e("eloop:")
+    e("  setp.lt.u s7, s6, s5")
+    e("  brz s7, vnext")
+    e("ebody:")
+    e("  iadd v0, s6, %laneid")
+    e("  setp.lt.u v1, v0, s5")
+    e("  @v1 ldg v2, colidx[v0]")                     # neighbour u
+    e("  poll")
+    e("  @v1 atom.cas v3, dist[v2], 0xFFFFFFFF, %lvl1")
+    e("  setp.eq.u v4, v3, 0xFFFFFFFF")
+    e("  and v4, v4, v1")                             # newly discovered
+    e("  @v4 atom.add v5, nextcnt[0], 1")
+    e("  @v4 stg nextf[v5], v2")
+    e("  iadd s6, s6, 32")
+    e("  bra eloop")
+    e("vnext:")
+    e("  iadd s0, s0, s1")
+    e("  bra vloop")
+    e("done:")
+    e("  exit")
+    return "\n".join(L) + "\n"
+
+
+def c4b_graph(n=1 << 22, avg_deg=16, seed=41):
+    """Uniform random directed graph in CSR: out-degrees ~ Poisson(avg_deg)
+    (i.e. ~avg_deg*n edges with uniformly random endpoints), destinations
+    uniform.  Source vertex 0."""
+    r = np.random.default_rng(seed)
+    deg = r.poisson(avg_deg, n).astype(np.uint64)
+    rowptr = np.zeros(n + 1, dtype=np.uint64)
+    np.cumsum(deg, out=rowptr[1:])
+    m = int(rowptr[-1])
+    colidx = r.integers(0, n, m, dtype=np.uint64).astype(np.uint32)
+    return rowptr.astype(np.uint32), colidx
+
+
+def bfs_reference(rowptr, colidx, src=0):
+    """Plain level-synchronous BFS (numpy) -> dist (0xFFFFFFFF unreached)."""
+    n = len(rowptr) - 1
+    dist = np.full(n, 0xFFFFFFFF, dtype=np.uint32)
+    dist[src] = 0
+    front = np.array([src], dtype=np.int64)
+    lvl = 0
+    rp = rowptr.astype(np.int64)
+    while len(front):
+        beg, end = rp[front], rp[front + 1]
+        cnt = end - beg
+        idx = np.repeat(beg - np.concatenate(([0], np.cumsum(cnt)[:-1])), cnt) + np.arange(cnt.sum())
+        nb = colidx[idx].astype(np.int64)
+        nb = np.unique(nb[dist[nb] == 0xFFFFFFFF])
+        lvl += 1
+        dist[nb] = lvl
+        front = nb
+    return dist
