@@ -50,20 +50,29 @@ def parse():
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-oracle", action="store_true")
     ap.add_argument("--seed", type=int, default=100)
+    ap.add_argument("--configs", default="c1,c3,c4a,c4b,c5",
+                    help="extra BASELINE configs measured after the C2 headline (comma list, or 'none')")
+    ap.add_argument("--config-trials", type=int, default=5)
+    ap.add_argument("--c5-seconds", type=float, default=4.0)
     return ap.parse_args()
 
 
 # ---- distributed plumbing (replicas only) ------------------------------------
 
-def dist_setup(args):
+def dist_setup(args=None, backend="nccl"):
+    """Replicas only: one process per GPU (RANK / LOCAL_RANK / WORLD_SIZE from
+    torchrun).  The process group carries nothing but the timing reduction."""
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if ws > 1:
         import torch
         import torch.distributed as dist
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            torch.cuda.set_device(local)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     return ws, rank, local
 
 
@@ -74,12 +83,26 @@ def barrier(ws):
 
 
 def allmax(ws, x):
+    """Max over ranks (the slowest replica's time is the job's time)."""
     if ws <= 1:
         return x
     import torch
     import torch.distributed as dist
-    t = torch.tensor([float(x)], device="cuda")
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([float(x)], device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def allsum(ws, x):
+    """Sum over ranks (aggregate throughput of the replicas, a sanity check)."""
+    if ws <= 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([float(x)], device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
     return float(t.item())
 
 
@@ -328,6 +351,468 @@ def oracle_sample(steps=1, seed=0):
     return out, t_an
 
 
+
+# ---- the other BASELINE configs (configs[0], [2], [3]) ----------------------
+
+MODES = (("ctxback", 0), ("full_hw", 3), ("live", 1))
+
+
+def _progs(cb, ir_text, debug=0, min_blocks=0):
+    return {name: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT if "poll" in ir_text else cb.POLL_EVERY_INSTR,
+                             mode=mode, debug=debug, min_blocks_per_sm=min_blocks)
+            for name, mode in MODES}
+
+
+def _grid(progs):
+    bps, nsm = None, None
+    for p in progs.values():
+        b, nsm = p.occupancy()
+        bps = b if bps is None else min(bps, b)
+    return bps * nsm
+
+
+def _static(prog, nwarps):
+    si = [prog.site_info(k) for k in range(prog.num_sites)]
+    return {"ctxback_bytes_per_tb_per_site": [nwarps * x["payload_bytes_per_warp"] for x in si],
+            "live_bytes_per_tb_per_site": [nwarps * x["live_bytes_per_warp"] for x in si],
+            "full_ir_bytes_per_tb": nwarps * prog.info["full_ir_bytes_per_warp"],
+            "revert_sites": sum(1 for x in si if x["n_revert_pre"] + x["n_revert_res"]),
+            "osrb_backups": len(prog.backups)}
+
+
+def _flag_trials(progs, grid, make_bufs, uniforms, check, fracs, T_s):
+    """For each mode: launch, flag at frac*T, resume, check outputs."""
+    import torch
+    s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
+    out = {}
+    for name, prog in progs.items():
+        ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+        recs = []
+        for fr in fracs:
+            bufs = make_bufs()
+            torch.cuda.synchronize()
+            run = prog.launch(grid, bufs, uniforms, ctx, s)
+            spin_until(time.perf_counter() + fr * T_s)
+            st = run.preempt(ctrl)
+            rs = {"resume_us": 0.0}
+            if st["warps_preempted"]:
+                run.resume(s)
+                run.wait()
+                rs = run.resume_stats()
+            torch.cuda.synchronize()
+            if not check(bufs):
+                raise SystemExit(f"{name}: output differs after preempt/resume")
+            recs.append(dict(latency_us=st["latency_us"], host_us=st["host_us"], resume_us=rs["resume_us"],
+                             payload=st["payload_bytes"], header=st["header_bytes"], blocks=st["blocks_preempted"],
+                             warps=st["warps_preempted"], done=st["warps_done"], step_ms=0.0, launches=2))
+            del run
+        out[name] = summarize(recs)
+    return out
+
+
+def _reduction(res):
+    c, f = res.get("ctxback", {}), res.get("full_hw", {})
+    def pct(k):
+        if c.get(k) and f.get(k):
+            return round(100 * (1 - c[k] / f[k]), 2)
+        return None
+    return {"latency_pct": pct("latency_us_median"), "resume_pct": pct("resume_us_median"),
+            "context_pct": pct("context_bytes_per_tb")}
+
+
+def bench_c1(cb):
+    """C1 (configs[0]): 24-instruction kernel, 1 TB x 128 threads, preempted at
+    every site (forced mode, all 4 warps); device latency / resume per site."""
+    import torch
+    from workloads import configs
+    cfg = configs.c1()
+    names = ["in0", "in1", "rw0", "out"]
+    res = {}
+    for name, mode in MODES:
+        prog = cb.Program(cfg["ir"], mode=mode, debug=cb.DEBUG_FORCED)
+        ctx = torch.zeros(prog.context_capacity(1), dtype=torch.uint8, device="cuda")
+        dev = {n: torch.from_numpy(cfg["buffers"][n].view(np.int32).copy()).cuda() for n in names}
+        ref = None
+        recs = []
+        for k in range(-1, prog.num_sites):
+            dev["out"].zero_()
+            t = np.full(4, cb.NEVER if k < 0 else k, np.uint32)
+            run = prog.launch(1, [dev[n] for n in names], [], ctx, forced=t)
+            fin = run.wait()
+            if k >= 0:
+                assert not fin
+                pb, hb, _ = run.context_bytes()
+                st = run.stamps()
+                lat = (st[:, 1].max() - st[:, 0].min()) / 1e3
+                run.resume(forced=np.full(4, cb.NEVER, np.uint32))
+                assert run.wait()
+                rs = run.resume_stats()
+                recs.append(dict(latency_us=float(lat), resume_us=rs["resume_us"], payload=pb, header=hb,
+                                 blocks=1, warps=4, done=0, host_us=0.0, step_ms=0.0, launches=2))
+            out = dev["out"].cpu().numpy().view(np.uint32).copy()
+            if ref is None:
+                ref = out
+            elif not np.array_equal(out, ref):
+                raise SystemExit("C1 output differs after preempt/resume")
+            del run
+        res[name] = summarize(recs)
+        if name == "ctxback":
+            res["static"] = _static(prog, 4)
+    res["reduction_vs_full_hw"] = _reduction(res)
+    res["workload"] = "C1 24-instruction IR kernel, 1 TB x 128 threads, all warps preempted at each of the 24 sites"
+    return res
+
+
+def bench_c3(cb, trials, seed):
+    import torch
+    from workloads import configs
+    cfg = configs.c3()
+    W, H = cfg["W"], cfg["H"]
+    progs = _progs(cb, cfg["ir"])
+    grid = _grid(progs)
+    dX = torch.from_numpy(cfg["buffers"]["X"].view(np.int32)).cuda()
+    dY = torch.zeros(W * H, dtype=torch.int32, device="cuda")
+    ctx = torch.empty(progs["ctxback"].context_capacity(grid), dtype=torch.uint8, device="cuda")
+    run = progs["ctxback"].launch(grid, [dX, dY], [], ctx)
+    run.wait()
+    T = run.launch_ms()
+    ref = dY.clone()
+    del run
+    ok = np.array_equal(ref.cpu().numpy().view(np.uint32), configs.c3_numpy_reference(cfg["buffers"]["X"], W, H))
+
+    def make():
+        dY.zero_()
+        return [dX, dY]
+    fr = np.random.default_rng(seed + 2).uniform(0.05, 0.95, trials)
+    res = _flag_trials(progs, grid, make, [], lambda b: bool(torch.equal(b[1], ref)), fr, T / 1e3)
+    res["static"] = _static(progs["ctxback"], 8)
+    res["reduction_vs_full_hw"] = _reduction(res)
+    res["t_uninterrupted_ms"] = round(T, 3)
+    res["grid"] = grid
+    res["uninterrupted_equals_numpy"] = ok
+    res["workload"] = f"C3 5-point stencil IR {W}x{H} f32, persistent grid, flag at U[0.05,0.95] x T"
+    return res
+
+
+def bench_c4a(cb, trials, seed):
+    import torch
+    from workloads import configs
+    cfg = configs.c4a(1 << 28, grid=1)
+    progs = _progs(cb, cfg["ir"])
+    grid = _grid(progs)
+    keys = cfg["buffers"]["keys"]
+    want = torch.from_numpy(np.bincount(keys >> 24, minlength=256).astype(np.int32)).cuda()
+    dK = torch.from_numpy(keys.view(np.int32)).cuda()
+    dS = torch.from_numpy(cfg["buffers"]["starts"].view(np.int32)).cuda()
+    dH = torch.zeros(256 * grid, dtype=torch.int32, device="cuda")
+    hsum = lambda h: h.view(grid, 256).sum(0, dtype=torch.int64).to(torch.int32)  # noqa: E731
+    ctx = torch.empty(progs["ctxback"].context_capacity(grid), dtype=torch.uint8, device="cuda")
+    run = progs["ctxback"].launch(grid, [dK, dS, dH], [], ctx)
+    run.wait()
+    T = run.launch_ms()
+    ok = bool(torch.equal(hsum(dH), want))
+    del run
+
+    def make():
+        dH.zero_()
+        return [dK, dS, dH]
+    fr = np.random.default_rng(seed + 3).uniform(0.05, 0.95, trials)
+    res = _flag_trials(progs, grid, make, [], lambda b: bool(torch.equal(hsum(b[2]), want)), fr, T / 1e3)
+    res["static"] = _static(progs["ctxback"], 8)
+    osrb_off = cb.Program(cfg["ir"], flags=cb.RELAXED | cb.REVERT, poll_policy=cb.POLL_EXPLICIT,
+                          debug=cb.DEBUG_NO_COMPILE)
+    res["static"]["ctxback_osrb_off_bytes_per_tb_per_site"] = [
+        8 * osrb_off.site_info(k)["payload_bytes_per_warp"] for k in range(osrb_off.num_sites)]
+    res["reduction_vs_full_hw"] = _reduction(res)
+    res["t_uninterrupted_ms"] = round(T, 3)
+    res["grid"] = grid
+    res["uninterrupted_equals_bincount"] = ok
+    res["workload"] = ("C4a 256-bin histogram IR, 2^28 uniform u32 keys (1 GiB), global atomics into per-block "
+                       "bin copies, flag at U[0.05,0.95] x T")
+    return res
+
+
+def bench_c4b(cb, trials, seed):
+    import torch
+    from workloads import configs
+    rp, ci = configs.c4b_graph()
+    n = len(rp) - 1
+    want = configs.bfs_reference(rp, ci)
+    ir_text = configs.c4b_ir()
+    progs = _progs(cb, ir_text)
+    grid = _grid(progs)
+    d_rp = torch.from_numpy(rp.view(np.int32)).cuda()
+    d_ci = torch.from_numpy(ci.view(np.int32)).cuda()
+    want_t = torch.from_numpy(want.view(np.int32)).cuda()
+    fronts = [torch.zeros(n + 1, dtype=torch.int32, device="cuda") for _ in range(2)]
+    d_dist = torch.empty(n, dtype=torch.int32, device="cuda")
+    cnt = torch.zeros(1, dtype=torch.int32, device="cuda")
+    s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
+    # level sizes / durations from an uninterrupted run
+    sizes = np.bincount(want[want != 0xFFFFFFFF].astype(np.int64))
+    big = int(np.argmax(sizes))            # level whose kernel processes the largest frontier
+    res = {}
+    rng = np.random.default_rng(seed + 4)
+    for name, prog in progs.items():
+        ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+        recs = []
+        Tbig = None
+        for trial in range(trials + 1):
+            d_dist.fill_(-1)
+            d_dist[0] = 0
+            fronts[0][0] = 0
+            nf, lvl = 1, 0
+            while nf:
+                cnt.zero_()
+                torch.cuda.synchronize()
+                bufs = [d_rp, d_ci, fronts[lvl % 2], d_dist, fronts[(lvl + 1) % 2], cnt]
+                run = prog.launch(grid, bufs, [nf, lvl + 1], ctx, s)
+                if lvl == big and trial > 0:
+                    spin_until(time.perf_counter() + rng.uniform(0.05, 0.95) * Tbig)
+                    st = run.preempt(ctrl)
+                    rs = {"resume_us": 0.0}
+                    if st["warps_preempted"]:
+                        run.resume(s)
+                        run.wait()
+                        rs = run.resume_stats()
+                    recs.append(dict(latency_us=st["latency_us"], host_us=st["host_us"], resume_us=rs["resume_us"],
+                                     payload=st["payload_bytes"], header=st["header_bytes"],
+                                     blocks=st["blocks_preempted"], warps=st["warps_preempted"],
+                                     done=st["warps_done"], step_ms=0.0, launches=2))
+                else:
+                    run.wait()
+                    if lvl == big and trial == 0:
+                        Tbig = run.launch_ms() / 1e3
+                del run
+                nf = int(cnt.item())
+                lvl += 1
+            if not torch.equal(d_dist, want_t):
+                raise SystemExit(f"C4b {name}: dist differs from the reference BFS")
+        res[name] = summarize(recs)
+    res["static"] = _static(progs["ctxback"], 8)
+    res["reduction_vs_full_hw"] = _reduction(res)
+    res["grid"] = grid
+    res["largest_level"] = big
+    res["workload"] = (f"C4b level-synchronous BFS IR, n=2^22, {len(ci)} edges (Poisson(16) out-degree), "
+                       f"preempted at U[0.05,0.95] x T in the largest level")
+    return res
+
+def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
+    """C5 (configs[4]): batch jobs C2, C3, C4a, C4b back to back at full
+    occupancy; latency-sensitive (LS) jobs arrive Poisson (mean 10 ms) and each
+    runs a ~1.5 ms full-GPU cuBLAS GEMM on a high-priority stream.  Per arrival:
+    ctxb_preempt the running batch kernel -> LS -> ctxb_resume ("none": no
+    preemption, the LS job waits for the SMs).  Every batch output is checked
+    bit-exact.  Reports LS waiting time (arrival -> LS start), device
+    preemption latency, resume time and batch throughput vs no arrivals."""
+    import torch
+    from workloads import configs
+    s = torch.cuda.Stream()
+    ctrl = torch.cuda.Stream()
+    hp = torch.cuda.Stream(priority=-1)
+    # ---- LS job: calibrated to ~1.5 ms ----
+    ls_a = torch.randn(8192, 8192, device="cuda", dtype=torch.bfloat16)
+    ls_b = torch.randn(8192, 8192, device="cuda", dtype=torch.bfloat16)
+    with torch.cuda.stream(hp):
+        for _ in range(3):
+            ls_c = ls_a @ ls_b
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with torch.cuda.stream(hp):
+        e0.record(hp)
+        ls_c = ls_a @ ls_b
+        e1.record(hp)
+    torch.cuda.synchronize()
+    reps = max(1, int(round(1.5 / e0.elapsed_time(e1))))
+
+    def ls_job():
+        with torch.cuda.stream(hp):
+            for _ in range(reps):
+                torch.matmul(ls_a, ls_b, out=ls_c)
+    with torch.cuda.stream(hp):
+        e0.record(hp)
+        ls_job()
+        e1.record(hp)
+    torch.cuda.synchronize()
+    ls_ms = e0.elapsed_time(e1)
+    # ---- batch jobs (inputs + references) ----
+    c2 = configs.c2()
+    c3 = configs.c3()
+    c4a = configs.c4a(1 << 28, grid=1)
+    rp, ci = configs.c4b_graph()
+    bfs_want = torch.from_numpy(configs.bfs_reference(rp, ci).view(np.int32)).cuda()
+    n = len(rp) - 1
+    T = {}
+    dev = {
+        "A": torch.from_numpy(c2["buffers"]["A"].view(np.int32)).cuda(),
+        "B": torch.from_numpy(c2["buffers"]["B"].view(np.int32)).cuda(),
+        "C": torch.zeros(4096 * 4096, dtype=torch.int32, device="cuda"),
+        "X": torch.from_numpy(c3["buffers"]["X"].view(np.int32)).cuda(),
+        "Y": torch.zeros(c3["W"] * c3["H"], dtype=torch.int32, device="cuda"),
+        "keys": torch.from_numpy(c4a["buffers"]["keys"].view(np.int32)).cuda(),
+        "starts": torch.from_numpy(c4a["buffers"]["starts"].view(np.int32)).cuda(),
+        "rp": torch.from_numpy(rp.view(np.int32)).cuda(), "ci": torch.from_numpy(ci.view(np.int32)).cuda(),
+        "dist": torch.empty(n, dtype=torch.int32, device="cuda"),
+        "f0": torch.zeros(n + 1, dtype=torch.int32, device="cuda"),
+        "f1": torch.zeros(n + 1, dtype=torch.int32, device="cuda"),
+        "cnt": torch.zeros(1, dtype=torch.int32, device="cuda"),
+    }
+    hist_want = torch.from_numpy(np.bincount(c4a["buffers"]["keys"] >> 24, minlength=256).astype(np.int32)).cuda()
+    irs = {"c2": (configs.c2_ir(4096, 4096, 4096, polls="iter"), 2), "c3": (c3["ir"], 0),
+           "c4a": (c4a["ir"], 0), "c4b": (configs.c4b_ir(), 0)}
+    mode_id = {"ctxback": cb.MODE_CTXBACK, "full_hw": cb.MODE_FULL_HW, "none": cb.MODE_CTXBACK}
+    results = {}
+    refs = {}
+    for mode in modes:
+        progs, grids, ctxs = {}, {}, {}
+        for k, (txt, mb) in irs.items():
+            progs[k] = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, mode=mode_id[mode], min_blocks_per_sm=mb)
+            b_, nsm = progs[k].occupancy()
+            grids[k] = b_ * nsm
+            ctxs[k] = torch.empty(progs[k].context_capacity(grids[k]), dtype=torch.uint8, device="cuda")
+        dev["H"] = torch.zeros(256 * grids["c4a"], dtype=torch.int32, device="cuda")
+
+        class Job:
+            def __init__(self, kind):
+                self.kind = kind
+                self.lvl = 0
+                self.nf = 1
+                if kind == "c2":
+                    dev["C"].zero_()
+                elif kind == "c3":
+                    dev["Y"].zero_()
+                elif kind == "c4a":
+                    dev["H"].zero_()
+                else:
+                    dev["dist"].fill_(-1)
+                    dev["dist"][0] = 0
+                    dev["f0"][0] = 0
+                self.run = None
+
+            def launch(self):
+                k = self.kind
+                if k == "c2":
+                    bufs, uni = [dev["A"], dev["B"], dev["C"]], []
+                elif k == "c3":
+                    bufs, uni = [dev["X"], dev["Y"]], []
+                elif k == "c4a":
+                    bufs, uni = [dev["keys"], dev["starts"], dev["H"]], []
+                else:
+                    dev["cnt"].zero_()
+                    fa, fb = (dev["f0"], dev["f1"]) if self.lvl % 2 == 0 else (dev["f1"], dev["f0"])
+                    bufs, uni = [dev["rp"], dev["ci"], fa, dev["dist"], fb, dev["cnt"]], [self.nf, self.lvl + 1]
+                self.run = progs[k].launch(grids[k], bufs, uni, ctxs[k], s)
+
+            def next_launch(self):
+                """After a completed launch: True if the job has more launches."""
+                if self.kind != "c4b":
+                    return False
+                self.nf = int(dev["cnt"].item())
+                self.lvl += 1
+                return self.nf > 0
+
+            def check(self):
+                k = self.kind
+                if k == "c2":
+                    return bool(torch.equal(dev["C"], refs["c2"]))
+                if k == "c3":
+                    return bool(torch.equal(dev["Y"], refs["c3"]))
+                if k == "c4a":
+                    return bool(torch.equal(dev["H"].view(-1, 256).sum(0, dtype=torch.int64).to(torch.int32),
+                                            hist_want))
+                return bool(torch.equal(dev["dist"], bfs_want))
+
+        if not refs:
+            for k in ("c2", "c3"):
+                j = Job(k)
+                j.launch()
+                j.run.wait()
+                refs[k] = (dev["C"] if k == "c2" else dev["Y"]).clone()
+        kinds = ["c2", "c3", "c4a", "c4b"]
+
+        def loop(arrivals, duration):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            ai, ji = 0, 0
+            job = Job(kinds[ji % 4])
+            job.launch()
+            done_jobs = {k: 0 for k in kinds}
+            recs = []
+            bad = 0
+            while True:
+                now = time.perf_counter() - t0
+                if ai < len(arrivals) and arrivals[ai] <= now:
+                    t_arr = arrivals[ai]
+                    ai += 1
+                    st = None
+                    tp0 = time.perf_counter()
+                    if mode != "none" and job.run is not None and job.run.running():
+                        st = job.run.preempt(ctrl)
+                    tp1 = time.perf_counter()
+                    with torch.cuda.stream(hp):
+                        le0 = torch.cuda.Event(enable_timing=True)
+                        le0.record(hp)
+                    t_ls = time.perf_counter() - t0
+                    ls_job()
+                    hp.synchronize()
+                    t_ls_done = time.perf_counter() - t0
+                    recs.append(dict(arr=t_arr, wait_ms=(t_ls_done - t_arr) * 1e3 - ls_ms,
+                                     host_to_ls_ms=(t_ls - t_arr) * 1e3, late_ms=(now - t_arr) * 1e3,
+                                     preempt_call_ms=(tp1 - tp0) * 1e3, kind=job.kind,
+                                     lat_us=st["latency_us"] if st and st["warps_preempted"] else None,
+                                     bytes=st["payload_bytes"] if st else 0,
+                                     blocks=st["blocks_preempted"] if st else 0))
+                    if st and st["warps_preempted"]:
+                        job.run.resume(s)
+                    continue
+                if job.run.running():
+                    continue
+                if not job.run.finished:      # preempted by us and not yet resumed: cannot happen
+                    job.run.resume(s)
+                    continue
+                if job.next_launch():
+                    job.launch()
+                    continue
+                if not job.check():
+                    bad += 1
+                done_jobs[job.kind] += 1
+                if now >= duration:
+                    break
+                ji += 1
+                job = Job(kinds[ji % 4])
+                job.launch()
+            wall = time.perf_counter() - t0
+            return recs, done_jobs, wall, bad
+
+        loop([], 0.3)                                           # warm-up
+        base_recs, base_done, base_wall, bad0 = loop([], seconds / 2)
+        arr = configs.c5_arrivals(seconds, 10.0, 51 + rank)
+        recs, done, wall, bad = loop(arr, seconds)
+        waits = np.array([r["wait_ms"] for r in recs]) if recs else np.zeros(1)
+        lats = np.array([r["lat_us"] for r in recs if r["lat_us"] is not None]) if recs else np.zeros(0)
+        jobs_base = sum(base_done.values()) / base_wall
+        jobs_trace = sum(done.values()) / wall
+        busy = len(recs) * ls_ms / 1e3 / wall
+        results[mode] = {
+            "arrivals": len(recs), "preemptions": int(len(lats)),
+            "ls_wait_ms_p50": float(np.median(waits)), "ls_wait_ms_p99": float(np.percentile(waits, 99)),
+            "ls_wait_ms_max": float(waits.max()),
+            "latency_us_p50": float(np.median(lats)) if len(lats) else None,
+            "latency_us_p99": float(np.percentile(lats, 99)) if len(lats) else None,
+            "latency_us_max": float(lats.max()) if len(lats) else None,
+            "batch_jobs_per_s_no_arrivals": jobs_base, "batch_jobs_per_s_with_trace": jobs_trace,
+            "ls_busy_fraction": busy,
+            "batch_throughput_loss_pct": 100.0 * (1 - jobs_trace / max(1e-9, jobs_base * (1 - busy))),
+            "jobs_done": done, "outputs_bit_exact": bad == 0 and bad0 == 0,
+            "worst_arrivals": sorted(recs, key=lambda r: -r["wait_ms"])[:5],
+        }
+        if bad or bad0:
+            raise SystemExit(f"C5 {mode}: a batch output differs")
+    return {"ls_job_ms": ls_ms, "ls_gemm_reps": reps, "seconds": seconds, "modes": results,
+            "workload": "C5: C2, C3, C4a, C4b back to back at full occupancy; LS jobs Poisson(mean 10 ms), "
+                        "each a ~1.5 ms bf16 GEMM on a high-priority stream; per arrival preempt -> LS -> resume"}
+
+
 def gpu_arm(args):
     import torch
     import paper_conf_ipps_jiw21_b200 as cb
@@ -396,6 +881,15 @@ def gpu_arm(args):
     bulk = bulk_bandwidth(cb, args.bulk_mib)
     peak, peak_src = peaks()
     traffic = ncu_traffic()
+    extra_cfg = {}
+    wanted = [] if args.configs == "none" else [c.strip() for c in args.configs.split(",") if c.strip()]
+    for cname in wanted:
+        fn = {"c1": lambda: bench_c1(cb), "c3": lambda: bench_c3(cb, args.config_trials, args.seed),
+              "c4a": lambda: bench_c4a(cb, args.config_trials, args.seed),
+              "c4b": lambda: bench_c4b(cb, args.config_trials, args.seed),
+              "c5": lambda: bench_c5(cb, args.c5_seconds, args.seed, rank)}.get(cname)
+        if fn is not None:
+            extra_cfg[cname] = fn()
     # ---- e2e: public API with pinned host buffers, H2D/D2H inside the step ----
     hA = torch.from_numpy(cfg["buffers"]["A"].view(np.int32)).pin_memory()
     hB = torch.from_numpy(cfg["buffers"]["B"].view(np.int32)).pin_memory()
@@ -424,6 +918,9 @@ def gpu_arm(args):
     # ---- max over ranks ----
     value = allmax(ws, main["latency_us_median"])
     ms_per_step = allmax(ws, float(np.mean([r["step_ms"] for r in recs])))
+    c5_total = None
+    if "c5" in extra_cfg:
+        c5_total = allsum(ws, extra_cfg["c5"]["modes"]["ctxback"]["batch_jobs_per_s_with_trace"])
     launches = int(sum(r["launches"] for r in recs))
     if rank != 0:
         return None
@@ -463,7 +960,7 @@ def gpu_arm(args):
             "context_pct": (round(100 * (1 - main["context_bytes_per_tb"] / base["full_hw"]["context_bytes_per_tb"]), 2)
                             if "full_hw" in base and base["full_hw"].get("context_bytes_per_tb") and
                             main.get("context_bytes_per_tb") else None)},
-        "poll_overhead": ovh, "bulk": bulk,
+        "poll_overhead": ovh, "bulk": bulk, "configs": extra_cfg,
         "roofline": rf, "roofline_restore": rr,
         "cpu_baseline": cpu,
         "e2e": {"value": round(e2e_val, 3), "unit": "us",
@@ -471,6 +968,8 @@ def gpu_arm(args):
                         "memory and C copied back every step",
                 "h2d_bytes_per_step": 2 * M * K * 4, "d2h_bytes_per_step": M * N * 4},
         "gpu_launches": launches, "clocks": clocks,
+        "replicas": {"n": ws, "c5_aggregate_batch_jobs_per_s": c5_total,
+                     "note": "independent per-GPU instances; no data-path collective"},
         "parity": "C bit-exact vs the uninterrupted run in every step",
     }
     return line

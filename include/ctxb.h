@@ -199,6 +199,11 @@ int ctxb_resume(ctxb_run* run, void* stream, const uint32_t* forced_targets);
  * 0 if some warps were preempted (forced mode or a racing ctxb_preempt). */
 int ctxb_wait(ctxb_run* run, int* finished);
 
+/* Non-blocking: *running = 1 while the run's current launch is executing;
+ * once it has completed, the headers are collected (as ctxb_wait does) and
+ * *running = 0.  Lets a host scheduler poll a batch job between arrivals. */
+int ctxb_query(ctxb_run* run, int* running);
+
 /* Duration of the run's last kernel launch (normal or resume), from CUDA
  * events the library records immediately before and after cuLaunchKernel on
  * the launching stream.  Valid after ctxb_wait / ctxb_preempt returned. */

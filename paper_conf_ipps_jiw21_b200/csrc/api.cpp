@@ -562,6 +562,24 @@ int ctxb_wait(ctxb_run* r, int* finished) {
   return CTXB_OK;
 }
 
+int ctxb_query(ctxb_run* r, int* running) {
+  if (!r || !running) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  if (r->state != RUN_RUNNING) {
+    *running = 0;
+    return CTXB_OK;
+  }
+  CUresult q = driver().cuEventQuery(r->ev1);
+  if (q == CUDA_ERROR_NOT_READY) {
+    *running = 1;
+    return CTXB_OK;
+  }
+  if (q != CUDA_SUCCESS) return fail(CTXB_E_CUDA, "cuEventQuery: " + cu_err(q));
+  int rc = collect(r);
+  if (rc) return rc;
+  *running = 0;
+  return CTXB_OK;
+}
+
 int ctxb_launch_ms(const ctxb_run* r, float* ms) {
   if (!r || !ms) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   if (r->state == RUN_RUNNING) return fail(CTXB_E_STATE, "launch still running: call ctxb_wait/ctxb_preempt first");

@@ -50,7 +50,7 @@ Driver& driver() {
               sym(h, "cuEventCreate", &d.cuEventCreate, &e) && sym(h, "cuEventRecord", &d.cuEventRecord, &e) &&
               sym(h, "cuEventSynchronize", &d.cuEventSynchronize, &e) &&
               sym(h, "cuEventElapsedTime", &d.cuEventElapsedTime, &e) &&
-              sym(h, "cuEventDestroy_v2", &d.cuEventDestroy, &e);
+              sym(h, "cuEventDestroy_v2", &d.cuEventDestroy, &e) && sym(h, "cuEventQuery", &d.cuEventQuery, &e);
     if (ok && !sym(h, "cuStreamWriteValue32_v2", &d.cuStreamWriteValue32, &e))
       ok = sym(h, "cuStreamWriteValue32", &d.cuStreamWriteValue32, &e);
     if (!ok) return;

@@ -35,7 +35,7 @@ EXPORTED_SYMBOLS = [
     "ctxb_last_error", "ctxb_version", "ctxb_analyze", "ctxb_program_destroy", "ctxb_program_info",
     "ctxb_num_sites", "ctxb_site_info", "ctxb_backups", "ctxb_site_plan_text", "ctxb_generated_source",
     "ctxb_occupancy", "ctxb_context_capacity", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait",
-    "ctxb_launch_ms", "ctxb_resume_stats_get", "ctxb_context_bytes", "ctxb_read_headers", "ctxb_read_stamps",
+    "ctxb_query", "ctxb_launch_ms", "ctxb_resume_stats_get", "ctxb_context_bytes", "ctxb_read_headers", "ctxb_read_stamps",
     "ctxb_run_destroy",
 ]
 
@@ -99,6 +99,7 @@ def _load():
         "ctxb_wait": (I, [P, C.POINTER(I)]),
         "ctxb_resume_stats_get": (I, [P, C.POINTER(_ResStats)]),
         "ctxb_launch_ms": (I, [P, C.POINTER(C.c_float)]),
+        "ctxb_query": (I, [P, C.POINTER(I)]),
         "ctxb_context_bytes": (I, [P, C.POINTER(U64), C.POINTER(U64), C.POINTER(U32)]),
         "ctxb_read_headers": (I, [P, C.POINTER(U32), U64]),
         "ctxb_read_stamps": (I, [P, C.POINTER(U64), U64]),
@@ -277,6 +278,19 @@ class Run:
         _chk(lib.ctxb_resume(self._h, _stream(stream), f[1] if f else None))
 
     def wait(self):
+        fin = C.c_int()
+        _chk(lib.ctxb_wait(self._h, C.byref(fin)))
+        return bool(fin.value)
+
+    def running(self):
+        """Non-blocking: True while the current launch executes (ctxb_query)."""
+        r = C.c_int()
+        _chk(lib.ctxb_query(self._h, C.byref(r)))
+        return bool(r.value)
+
+    @property
+    def finished(self):
+        """After the current launch completed: every warp done (no preempted warp left)."""
         fin = C.c_int()
         _chk(lib.ctxb_wait(self._h, C.byref(fin)))
         return bool(fin.value)

@@ -62,7 +62,7 @@ def test_c3_small_forced():
 
 
 def test_c4a_small_forced():
-    cfg = configs.c4a(1 << 14)
+    cfg = configs.c4a(1 << 14, grid=2)
     an = forced_parity(cfg, 2, 3, 4)
     assert an.backups, "C4a must select an OSRB backup"
 
@@ -135,7 +135,7 @@ def test_c3_full_flag():
 def test_c4a_full_flag(skewed):
     import torch
     cb = _cb()
-    cfg = configs.c4a(1 << 28, skewed=skewed)
+    cfg = configs.c4a(1 << 28, skewed=skewed, grid=1)
     op = ir.parse(cfg["ir"])
     an = A.analyze(op, policy="EXPLICIT")
     prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT)
@@ -144,13 +144,14 @@ def test_c4a_full_flag(skewed):
     keys = cfg["buffers"]["keys"]
     want = np.bincount(keys >> 24, minlength=256).astype(np.uint32)
     dK, dS = to_dev(keys), to_dev(cfg["buffers"]["starts"])
-    dH = torch.zeros(256, dtype=torch.int32, device="cuda")
+    dH = torch.zeros(256 * grid, dtype=torch.int32, device="cuda")
+    total = lambda: from_dev(dH).reshape(grid, 256).astype(np.uint64).sum(0).astype(np.uint32)  # noqa: E731
     ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
     s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
     run = prog.launch(grid, [dK, dS, dH], [], ctx, s)
     assert run.wait()
     T = run.launch_ms() / 1e3
-    assert np.array_equal(from_dev(dH), want)
+    assert np.array_equal(total(), want)
     sb = [an.plans[c].payload_bytes for c in an.sites]
     lb = [an.live[c].payload_bytes for c in an.sites]
     for fr in (0.3, 0.7):
@@ -159,7 +160,7 @@ def test_c4a_full_flag(skewed):
         st, hdr, _ = flag_run(prog, grid, [dK, dS, dH], [], ctx, fr * T, s, ctrl)
         torch.cuda.synchronize()
         check_headers_vs_plans(hdr, 1, sb, lb)
-        assert np.array_equal(from_dev(dH), want)
+        assert np.array_equal(total(), want)
 
 
 def test_c4b_full_flag():

@@ -295,21 +295,24 @@ def c3_numpy_reference(x_bits, W, H):
 # configs[3]: "histogram + BFS-frontier IR kernels with scalar-operand-limited
 # re-execution (exercises on-chip scalar backup)".
 def c4a_ir(nkeys=1 << 28, per_lane=8):
-    """256-bin histogram of u32 keys (bin = key >> 24) with global atomics.
-    Warp-cooperative chunk loop: a warp handles chunks of 32*per_lane keys;
-    the chunk base is a scalar loaded from `starts` (an irreversible uniform
-    load that overwrites the base the chunk's key loads were addressed from --
-    the OSRB case).  One poll per chunk, after the next base is
-    loaded and before the atomics."""
+    """256-bin histogram of u32 keys (bin = key >> 24) with global atomics
+    into a per-block private copy of the bins (hist[ctaid*256 + bin]; the
+    copies are summed afterwards) so that atomics on the same address only
+    come from one block.  Warp-cooperative chunk loop: a warp handles chunks
+    of 32*per_lane keys; the chunk base is a scalar loaded from `starts` (an
+    irreversible uniform load that overwrites the base the chunk's key loads
+    were addressed from -- the OSRB case).  One poll per chunk,
+    after the next base is loaded and before the atomics."""
     chunk = 32 * per_lane
     assert nkeys % chunk == 0
     nch = nkeys // chunk
     L = [".kernel c4a_hist", ".buffer ro keys", ".buffer ro starts", ".buffer rw hist",
-         f".vregs {1 + 2 * per_lane}", ".sregs 6", ".block 256"]
+         f".vregs {1 + 2 * per_lane}", ".sregs 7", ".block 256"]
     e = L.append
     e("init:")
     e("  imad s0, %ctaid, %nwarps, %warpid")          # chunk index = global warp id
     e("  imul s1, %nctaid, %nwarps")                  # total warps
+    e("  shl s6, %ctaid, 8")                          # this block's private bins
     e(f"  setp.lt.u s2, s0, {nch}")
     e("  brz s2, done")
     e("first:")
@@ -322,6 +325,7 @@ def c4a_ir(nkeys=1 << 28, per_lane=8):
             e("  iadd v0, v0, 32")
     for j in range(per_lane):
         e(f"  shr v{1 + per_lane + j}, v{1 + j}, 24")
+        e(f"  iadd v{1 + per_lane + j}, v{1 + per_lane + j}, s6")
     e("  iadd s0, s0, s1")                            # next chunk (reversible)
     e(f"  setp.lt.u s2, s0, {nch}")
     e(f"  umin s4, s0, {nch - 1}")
@@ -335,7 +339,9 @@ def c4a_ir(nkeys=1 << 28, per_lane=8):
     return "\n".join(L) + "\n"
 
 
-def c4a(nkeys=1 << 28, skewed=False, per_lane=8):
+def c4a(nkeys=1 << 28, skewed=False, per_lane=8, grid=2):
+    """`grid` = number of blocks the kernel is launched with (the hist buffer
+    holds one 256-bin copy per block)."""
     chunk = 32 * per_lane
     if skewed:
         r = np.random.default_rng(32)
@@ -345,8 +351,8 @@ def c4a(nkeys=1 << 28, skewed=False, per_lane=8):
         r = np.random.default_rng(31)
         keys = r.integers(0, 1 << 32, nkeys, dtype=np.uint64).astype(np.uint32)
     starts = (np.arange(nkeys // chunk, dtype=np.uint64) * chunk).astype(np.uint32)
-    bufs = {"keys": keys, "starts": starts, "hist": np.zeros(256, dtype=np.uint32)}
-    return dict(name="C4a", ir=c4a_ir(nkeys, per_lane), grid=None, buffers=bufs, uniforms={},
+    bufs = {"keys": keys, "starts": starts, "hist": np.zeros(256 * grid, dtype=np.uint32)}
+    return dict(name="C4a", ir=c4a_ir(nkeys, per_lane), grid=grid, buffers=bufs, uniforms={},
                 policy="EXPLICIT", nkeys=nkeys, min_blocks=0)
 
 
@@ -427,3 +433,13 @@ def bfs_reference(rowptr, colidx, src=0):
         dist[nb] = lvl
         front = nb
     return dist
+
+
+# configs[4]: "full-occupancy mixed suite on 1 B200 under a latency-sensitive
+# arrival trace, plus 8 independent per-GPU instances".
+def c5_arrivals(seconds, mean_ms=10.0, seed=51):
+    """Poisson arrival times (s) of latency-sensitive jobs, mean gap mean_ms."""
+    r = np.random.default_rng(seed)
+    gaps = r.exponential(mean_ms / 1e3, int(seconds / (mean_ms / 1e3) * 3) + 16)
+    t = np.cumsum(gaps)
+    return t[t < seconds]
