@@ -187,12 +187,18 @@ def preempt_steps(cb, prog, grid, bufs, ctx, s, ctrl, ref, t_unint_s, fracs, ws,
         rs = {"resume_us": 0.0, "warps_resumed": 0}
         run_ms = run.launch_ms()
         res_ms = None
+        save_w = restore_w = None
         if st["warps_preempted"]:
+            hdr = run.headers().copy()
+            pre = (hdr[:, 2] == 1) & (hdr[:, 3] == 1)
             run.resume(s)
             run.wait()
             launches += 1
             rs = run.resume_stats()
             res_ms = run.launch_ms()
+            stp = run.stamps()[pre].astype(np.int64)
+            save_w = float(np.median(stp[:, 1] - stp[:, 0])) / 1e3
+            restore_w = float(np.median(stp[:, 3] - stp[:, 2])) / 1e3
         with torch.cuda.stream(s):
             ev1.record(s)
         torch.cuda.synchronize()
@@ -200,7 +206,8 @@ def preempt_steps(cb, prog, grid, bufs, ctx, s, ctrl, ref, t_unint_s, fracs, ws,
         recs.append(dict(frac=fr, latency_us=st["latency_us"], host_us=st["host_us"], resume_us=rs["resume_us"],
                          payload=st["payload_bytes"], header=st["header_bytes"], blocks=st["blocks_preempted"],
                          warps=st["warps_preempted"], done=st["warps_done"], step_ms=ev0.elapsed_time(ev1),
-                         run_ms=run_ms, resume_ms=res_ms, launches=launches, ok=ok))
+                         run_ms=run_ms, resume_ms=res_ms, launches=launches, ok=ok,
+                         save_warp_us=save_w, restore_warp_us=restore_w))
         if check and not ok:
             raise SystemExit("C differs from the uninterrupted run after preempt/resume")
         del run
@@ -218,6 +225,12 @@ def summarize(recs):
         "host_latency_us_median": float(np.median([r["host_us"] for r in pre])) if pre else 0.0,
         "preempted_steps": len(pre), "steps": len(recs),
     }
+    sw = [r["save_warp_us"] for r in pre if r.get("save_warp_us") is not None]
+    rw = [r["restore_warp_us"] for r in pre if r.get("restore_warp_us") is not None]
+    if sw:
+        out["save_routine_us_per_warp_median"] = float(np.median(sw))
+    if rw:
+        out["restore_routine_us_per_warp_median"] = float(np.median(rw))
     if pre:
         bpt = [r["payload"] / max(1, r["blocks"]) for r in pre]
         out["context_bytes_per_tb"] = float(np.median(bpt))
@@ -269,7 +282,7 @@ def bulk_bandwidth(cb, mib, reps=5):
                 save_bytes=save_bytes, restore_bytes=rest_bytes)
 
 
-def poll_overhead(cb, size, grid, bufs, reps=5):
+def poll_overhead(cb, size, grid, bufs, reps=20):
     import torch
     out = {}
     for name, dbg in (("polls", 0), ("no_polls", cb.DEBUG_NO_POLLS)):
@@ -826,6 +839,7 @@ def gpu_arm(args):
     if not args.no_baselines:
         progs["live"] = make_c2(cb, size, cb.MODE_LIVE)
         progs["full_hw"] = make_c2(cb, size, cb.MODE_FULL_HW)
+        progs["full_ir"] = make_c2(cb, size, cb.MODE_FULL)
     bps, nsm = progs["ctxback"].occupancy()
     for p in progs.values():
         bps = min(bps, p.occupancy()[0])
@@ -835,6 +849,7 @@ def gpu_arm(args):
     dC = torch.zeros(M * N, dtype=torch.int32, device="cuda")
     s = torch.cuda.Stream()
     ctrl = torch.cuda.Stream()
+    prop_med, prop_max = cb.ctxb_flag_propagation(ctrl, 20)
     ctxs = {k: torch.empty(p.context_capacity(grid), dtype=torch.uint8, device="cuda") for k, p in progs.items()}
     # uninterrupted reference + its duration
     pr = progs["ctxback"]
@@ -861,7 +876,7 @@ def gpu_arm(args):
     main = summarize(recs)
     # ---- baselines in the same framework (same fracs) ----
     base = {}
-    for k in ("full_hw", "live"):
+    for k in ("full_hw", "full_ir", "live"):
         if k in progs:
             preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_w[:1], ws)
             r = preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_t, ws)
@@ -950,6 +965,10 @@ def gpu_arm(args):
                    "grid": grid, "block": 256, "t_uninterrupted_ms": round(t_unint_ms, 3),
                    "l2": "inputs larger than L2 (A, B, C = 192 MiB > 126 MB)", "parallelism": f"replicas x{ws}"},
         "resume_us": round(main["resume_us_median"], 3),
+        "flag_propagation_us": {"median": round(prop_med, 3), "max": round(prop_max, 3),
+                                "what": "device clock: stamp kernel on the control stream -> cuStreamWriteValue32 "
+                                        "-> a spinning warp sees the flag (idle GPU, 20 trials)"},
+        "latency_incl_flag_propagation_us": round(value + prop_med, 3),
         "context_bytes_per_tb": main.get("context_bytes_per_tb"),
         "ctxback": main, "baselines": base, "static_context": static,
         "reduction_vs_full_hw": {

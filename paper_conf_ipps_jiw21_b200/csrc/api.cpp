@@ -580,6 +580,85 @@ int ctxb_query(ctxb_run* r, int* running) {
   return CTXB_OK;
 }
 
+// ---- flag propagation probe (measured separately) -------------
+namespace {
+const char* kProbeSrc = R"CUDA(
+typedef unsigned int u32; typedef unsigned long long u64;
+static __device__ __forceinline__ u64 gt() { u64 t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); return t; }
+static __device__ __forceinline__ u32 ldcv(const u32* p) { u32 v; asm volatile("ld.global.cv.u32 %0, [%1];" : "=r"(v) : "l"(p)); return v; }
+extern "C" __global__ void ctxb_probe_spin(const u32* flag, u64* out) {
+  u64 t0 = gt();
+  while (ldcv(flag) == 0u) { if (gt() - t0 > 2000000000ull) break; }
+  if (threadIdx.x == 0) out[1] = gt();
+}
+extern "C" __global__ void ctxb_probe_stamp(u64* out) { if (threadIdx.x == 0) out[0] = gt(); }
+)CUDA";
+
+struct Probe {
+  CUmodule mod = nullptr;
+  CUfunction spin = nullptr, stamp = nullptr;
+};
+}  // namespace
+
+int ctxb_flag_propagation(void* ctrl, uint32_t trials, double* median_us, double* max_us) {
+  if (!median_us || trials == 0) return fail(CTXB_E_INVALID_ARG, "bad argument");
+  CUcontext c;
+  int rc = ensure_ctx(&c);
+  if (rc) return rc;
+  static std::mutex mu;
+  static std::map<CUcontext, Probe> probes;
+  std::lock_guard<std::mutex> g(mu);
+  Probe& P = probes[c];
+  Driver& d = driver();
+  if (!P.mod) {
+    Nvrtc& n = nvrtc();
+    if (!n.ok) return fail(CTXB_E_NVRTC, n.err);
+    void* prog = nullptr;
+    if (n.CreateProgram(&prog, kProbeSrc, "probe.cu", 0, nullptr, nullptr)) return fail(CTXB_E_NVRTC, "probe");
+    const char* opts[] = {"--gpu-architecture=sm_100a"};
+    if (n.CompileProgram(prog, 1, opts)) {
+      n.DestroyProgram(&prog);
+      return fail(CTXB_E_NVRTC, "probe compile");
+    }
+    size_t cs = 0;
+    n.GetCUBINSize(prog, &cs);
+    std::vector<char> cubin(cs);
+    n.GetCUBIN(prog, cubin.data());
+    n.DestroyProgram(&prog);
+    CU(d.cuModuleLoadData(&P.mod, cubin.data()));
+    CU(d.cuModuleGetFunction(&P.spin, P.mod, "ctxb_probe_spin"));
+    CU(d.cuModuleGetFunction(&P.stamp, P.mod, "ctxb_probe_stamp"));
+  }
+  CUdeviceptr flag = 0, out = 0;
+  CU(d.cuMemAlloc(&flag, 256));
+  CU(d.cuMemAlloc(&out, 64));
+  std::vector<double> v;
+  CUstream spin_s = nullptr;   // legacy stream for the spinner; ctrl for stamp + flag
+  for (uint32_t t = 0; t < trials; t++) {
+    uint32_t zero = 0;
+    CU(d.cuMemcpyHtoD(flag, &zero, 4));
+    void* a1[] = {&flag, &out};
+    CU(d.cuLaunchKernel(P.spin, 1, 1, 1, 32, 1, 1, 0, spin_s, a1, nullptr));
+    double t0 = now_ms();
+    while (now_ms() < t0 + 0.2) {
+    }
+    void* a2[] = {&out};
+    CU(d.cuLaunchKernel(P.stamp, 1, 1, 1, 32, 1, 1, 0, (CUstream)ctrl, a2, nullptr));
+    CU(d.cuStreamWriteValue32((CUstream)ctrl, flag, 1u, 0));
+    CU(d.cuStreamSynchronize((CUstream)ctrl));
+    CU(d.cuStreamSynchronize(spin_s));
+    uint64_t ts[2];
+    CU(d.cuMemcpyDtoH(ts, out, 16));
+    v.push_back((double)(int64_t)(ts[1] - ts[0]) * 1e-3);
+  }
+  d.cuMemFree(flag);
+  d.cuMemFree(out);
+  std::sort(v.begin(), v.end());
+  *median_us = v[v.size() / 2];
+  if (max_us) *max_us = v.back();
+  return CTXB_OK;
+}
+
 int ctxb_launch_ms(const ctxb_run* r, float* ms) {
   if (!r || !ms) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   if (r->state == RUN_RUNNING) return fail(CTXB_E_STATE, "launch still running: call ctxb_wait/ctxb_preempt first");

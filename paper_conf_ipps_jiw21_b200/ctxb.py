@@ -19,6 +19,7 @@ __all__ = [
     "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "EXPORTED_SYMBOLS",
     "ctxb_analyze", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait", "ctxb_context_bytes",
+    "ctxb_flag_propagation",
     "Program", "Run",
 ]
 
@@ -35,7 +36,7 @@ EXPORTED_SYMBOLS = [
     "ctxb_last_error", "ctxb_version", "ctxb_analyze", "ctxb_program_destroy", "ctxb_program_info",
     "ctxb_num_sites", "ctxb_site_info", "ctxb_backups", "ctxb_site_plan_text", "ctxb_generated_source",
     "ctxb_occupancy", "ctxb_context_capacity", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait",
-    "ctxb_query", "ctxb_launch_ms", "ctxb_resume_stats_get", "ctxb_context_bytes", "ctxb_read_headers", "ctxb_read_stamps",
+    "ctxb_query", "ctxb_flag_propagation", "ctxb_launch_ms", "ctxb_resume_stats_get", "ctxb_context_bytes", "ctxb_read_headers", "ctxb_read_stamps",
     "ctxb_run_destroy",
 ]
 
@@ -100,6 +101,7 @@ def _load():
         "ctxb_resume_stats_get": (I, [P, C.POINTER(_ResStats)]),
         "ctxb_launch_ms": (I, [P, C.POINTER(C.c_float)]),
         "ctxb_query": (I, [P, C.POINTER(I)]),
+        "ctxb_flag_propagation": (I, [P, U32, C.POINTER(C.c_double), C.POINTER(C.c_double)]),
         "ctxb_context_bytes": (I, [P, C.POINTER(U64), C.POINTER(U64), C.POINTER(U32)]),
         "ctxb_read_headers": (I, [P, C.POINTER(U32), U64]),
         "ctxb_read_stamps": (I, [P, C.POINTER(U64), U64]),
@@ -168,6 +170,14 @@ def ctxb_wait(run):
 
 def ctxb_context_bytes(run):
     return run.context_bytes()
+
+
+def ctxb_flag_propagation(ctrl_stream, trials=20):
+    """(median, max) us from the flag write on ctrl_stream to a spinning warp
+    seeing it (device clock)."""
+    m, x = C.c_double(), C.c_double()
+    _chk(lib.ctxb_flag_propagation(_stream(ctrl_stream), trials, C.byref(m), C.byref(x)))
+    return m.value, x.value
 
 
 class Program:
