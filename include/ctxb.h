@@ -204,12 +204,13 @@ int ctxb_wait(ctxb_run* run, int* finished);
  * *running = 0.  Lets a host scheduler poll a batch job between arrivals. */
 int ctxb_query(ctxb_run* run, int* running);
 
-/* Device-clock propagation time of the preemption signal: a one-warp
- * spinner polls a flag (ld.global.cv); a stamp kernel on `ctrl` records
- * %globaltimer and the flag is then written by cuStreamWriteValue32 on `ctrl`
- * (exactly as ctxb_preempt does); result = t(spinner saw flag) - t(stamp).
- * Median / max over `trials` (added to the drain latency as a
- * separately measured constant).  Needs an idle GPU. */
+/* Propagation time of the preemption signal: a one-warp spinner polls a flag
+ * (ld.relaxed.gpu, like the poll sites); an event is recorded on `ctrl` right
+ * before the flag is written by cuStreamWriteValue32 on `ctrl` (exactly as
+ * ctxb_preempt does) and another after the spinner on its own stream; result
+ * = elapsed time between the two (an upper bound: includes the spinner's
+ * exit).  Median / max over `trials` (added to the drain
+ * latency as a separately measured constant).  Needs an idle GPU. */
 int ctxb_flag_propagation(void* ctrl_stream, uint32_t trials, double* median_us, double* max_us);
 
 /* Duration of the run's last kernel launch (normal or resume), from CUDA

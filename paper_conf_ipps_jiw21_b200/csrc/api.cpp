@@ -211,7 +211,7 @@ int compile(ctxb_program* p) {
 void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>& blob) {
   size_t nb = std::max<size_t>(1, p->prog.buf_names.size());
   size_t nu = std::max<size_t>(1, p->prog.uniforms.size());
-  size_t words = nb + 5 + (nu + 4 + 1) / 2;
+  size_t words = nb + 5 + (nu + 5 + 1) / 2;
   blob.assign(words, 0);
   for (size_t i = 0; i < r->bufs.size(); i++) blob[i] = r->bufs[i];
   blob[nb + 0] = r->cbuf;
@@ -225,6 +225,7 @@ void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>
   u[nu + 1] = (uint32_t)r->stride;
   u[nu + 2] = p->pad_regs();
   u[nu + 3] = p->full_hw_bytes();
+  u[nu + 4] = 0;   // `zero`: opaque 0 for the timing dependency (gtimer_after)
 }
 
 int upload_forced(ctxb_run* r, const uint32_t* targets) {
@@ -260,7 +261,8 @@ int collect(ctxb_run* r) {
   Driver& d = driver();
   r->hdr_prev.swap(r->hdr);
   r->hdr.assign((size_t)r->n_warps * 4, 0);
-  CU(d.cuMemcpyDtoH(r->hdr.data(), r->cbuf, (size_t)r->n_warps * 16));
+  CU(d.cuMemcpyDtoHAsync(r->hdr.data(), r->cbuf, (size_t)r->n_warps * 16, r->stream));
+  CU(d.cuStreamSynchronize(r->stream));
   uint32_t pre = 0, done = 0;
   for (uint32_t w = 0; w < r->n_warps; w++) {
     const uint32_t* h = &r->hdr[(size_t)w * 4];
@@ -585,7 +587,7 @@ namespace {
 const char* kProbeSrc = R"CUDA(
 typedef unsigned int u32; typedef unsigned long long u64;
 static __device__ __forceinline__ u64 gt() { u64 t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); return t; }
-static __device__ __forceinline__ u32 ldcv(const u32* p) { u32 v; asm volatile("ld.global.cv.u32 %0, [%1];" : "=r"(v) : "l"(p)); return v; }
+static __device__ __forceinline__ u32 ldcv(const u32* p) { u32 v; asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p)); return v; }
 extern "C" __global__ void ctxb_probe_spin(const u32* flag, u64* out) {
   u64 t0 = gt();
   while (ldcv(flag) == 0u) { if (gt() - t0 > 2000000000ull) break; }
@@ -632,25 +634,49 @@ int ctxb_flag_propagation(void* ctrl, uint32_t trials, double* median_us, double
   CUdeviceptr flag = 0, out = 0;
   CU(d.cuMemAlloc(&flag, 256));
   CU(d.cuMemAlloc(&out, 64));
+  {
+    // load both kernels now (CUDA lazy loading would otherwise load the stamp
+    // kernel while the spinner runs, which waits for the spinner: deadlock)
+    uint32_t one = 1;
+    CU(d.cuMemcpyHtoD(flag, &one, 4));
+    void* a1[] = {&flag, &out};
+    CU(d.cuLaunchKernel(P.spin, 1, 1, 1, 32, 1, 1, 0, nullptr, a1, nullptr));
+    void* a2[] = {&out};
+    CU(d.cuLaunchKernel(P.stamp, 1, 1, 1, 32, 1, 1, 0, nullptr, a2, nullptr));
+    CU(d.cuStreamSynchronize(nullptr));
+  }
   std::vector<double> v;
-  CUstream spin_s = nullptr;   // legacy stream for the spinner; ctrl for stamp + flag
+  // The spinner runs on a private non-blocking stream.  Kernels on different
+  // streams are not guaranteed to be co-scheduled, so no stamp kernel is put
+  // in front of the flag write; instead an event on `ctrl` is recorded right
+  // before the write and one on the spinner's stream right after the
+  // spinner: elapsed = write issued -> spinner saw the flag and exited
+  // (an upper bound; includes the kernel's exit).
+  CUstream spin_s = nullptr;
+  CU(d.cuStreamCreate(&spin_s, CU_STREAM_NON_BLOCKING));
+  CUevent e0, e1;
+  CU(d.cuEventCreate(&e0, CU_EVENT_DEFAULT));
+  CU(d.cuEventCreate(&e1, CU_EVENT_DEFAULT));
   for (uint32_t t = 0; t < trials; t++) {
     uint32_t zero = 0;
     CU(d.cuMemcpyHtoD(flag, &zero, 4));
     void* a1[] = {&flag, &out};
     CU(d.cuLaunchKernel(P.spin, 1, 1, 1, 32, 1, 1, 0, spin_s, a1, nullptr));
+    CU(d.cuEventRecord(e1, spin_s));
     double t0 = now_ms();
     while (now_ms() < t0 + 0.2) {
     }
-    void* a2[] = {&out};
-    CU(d.cuLaunchKernel(P.stamp, 1, 1, 1, 32, 1, 1, 0, (CUstream)ctrl, a2, nullptr));
+    CU(d.cuEventRecord(e0, (CUstream)ctrl));
     CU(d.cuStreamWriteValue32((CUstream)ctrl, flag, 1u, 0));
     CU(d.cuStreamSynchronize((CUstream)ctrl));
     CU(d.cuStreamSynchronize(spin_s));
-    uint64_t ts[2];
-    CU(d.cuMemcpyDtoH(ts, out, 16));
-    v.push_back((double)(int64_t)(ts[1] - ts[0]) * 1e-3);
+    float ms = 0;
+    CU(d.cuEventElapsedTime(&ms, e0, e1));
+    v.push_back((double)ms * 1e3);
   }
+  d.cuEventDestroy(e0);
+  d.cuEventDestroy(e1);
+  d.cuStreamDestroy(spin_s);
   d.cuMemFree(flag);
   d.cuMemFree(out);
   std::sort(v.begin(), v.end());

@@ -50,7 +50,9 @@ Driver& driver() {
               sym(h, "cuEventCreate", &d.cuEventCreate, &e) && sym(h, "cuEventRecord", &d.cuEventRecord, &e) &&
               sym(h, "cuEventSynchronize", &d.cuEventSynchronize, &e) &&
               sym(h, "cuEventElapsedTime", &d.cuEventElapsedTime, &e) &&
-              sym(h, "cuEventDestroy_v2", &d.cuEventDestroy, &e) && sym(h, "cuEventQuery", &d.cuEventQuery, &e);
+              sym(h, "cuEventDestroy_v2", &d.cuEventDestroy, &e) && sym(h, "cuEventQuery", &d.cuEventQuery, &e) &&
+              sym(h, "cuStreamCreate", &d.cuStreamCreate, &e) && sym(h, "cuStreamDestroy_v2", &d.cuStreamDestroy, &e) &&
+              sym(h, "cuMemcpyDtoHAsync_v2", &d.cuMemcpyDtoHAsync, &e);
     if (ok && !sym(h, "cuStreamWriteValue32_v2", &d.cuStreamWriteValue32, &e))
       ok = sym(h, "cuStreamWriteValue32", &d.cuStreamWriteValue32, &e);
     if (!ok) return;

@@ -31,7 +31,7 @@ else:
     mb = 2
 bufs = mk()
 s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
-for name, mode in (("ctxback", 0), ("full_hw", 3), ("live", 1)):
+for name, mode in (("ctxback", 0), ("full_hw", 3), ("full_ir", 2), ("live", 1)):
     prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, mode=mode, min_blocks_per_sm=mb)
     bps, nsm = prog.occupancy()
     grid = bps * nsm
