@@ -118,13 +118,22 @@ class Clocks:
         self.gpu = gpu
         self.p = None
 
-    def start(self):
+    def start(self, wait_s=5.0):
+        """Start sampling and wait until the first sample is written, so the
+        timed region that follows is covered."""
         try:
             self.p = subprocess.Popen(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.Q}",
                                        "--format=csv,noheader,nounits", "-lms", "100"],
                                       stdout=self.f, stderr=subprocess.DEVNULL)
         except Exception:
             self.p = None
+            return
+        t0 = time.time()
+        while time.time() < t0 + wait_s:
+            self.f.flush()
+            if os.path.getsize(self.f.name) > 0:
+                break
+            time.sleep(0.05)
 
     def stop(self):
         if self.p is None:
@@ -203,7 +212,8 @@ def preempt_steps(cb, prog, grid, bufs, ctx, s, ctrl, ref, t_unint_s, fracs, ws,
             ev1.record(s)
         torch.cuda.synchronize()
         ok = bool(torch.equal(dC, ref)) if check else True
-        recs.append(dict(frac=fr, latency_us=st["latency_us"], host_us=st["host_us"], resume_us=rs["resume_us"],
+        recs.append(dict(frac=fr, latency_us=st["latency_us"], host_us=st["host_us"],
+                         signal_us=st["signal_to_drained_us"], resume_us=rs["resume_us"],
                          payload=st["payload_bytes"], header=st["header_bytes"], blocks=st["blocks_preempted"],
                          warps=st["warps_preempted"], done=st["warps_done"], step_ms=ev0.elapsed_time(ev1),
                          run_ms=run_ms, resume_ms=res_ms, launches=launches, ok=ok,
@@ -223,6 +233,8 @@ def summarize(recs):
         "latency_us_max": float(lat.max()),
         "resume_us_median": float(np.median(res)), "resume_us_max": float(res.max()),
         "host_latency_us_median": float(np.median([r["host_us"] for r in pre])) if pre else 0.0,
+        "signal_to_drained_us_median": (float(np.median([r["signal_us"] for r in pre if r.get("signal_us") is not None]))
+                                        if any(r.get("signal_us") is not None for r in pre) else None),
         "preempted_steps": len(pre), "steps": len(recs),
     }
     sw = [r["save_warp_us"] for r in pre if r.get("save_warp_us") is not None]
@@ -415,7 +427,8 @@ def _flag_trials(progs, grid, make_bufs, uniforms, check, fracs, T_s):
             torch.cuda.synchronize()
             if not check(bufs):
                 raise SystemExit(f"{name}: output differs after preempt/resume")
-            recs.append(dict(latency_us=st["latency_us"], host_us=st["host_us"], resume_us=rs["resume_us"],
+            recs.append(dict(latency_us=st["latency_us"], host_us=st["host_us"], signal_us=st["signal_to_drained_us"],
+                             resume_us=rs["resume_us"],
                              payload=st["payload_bytes"], header=st["header_bytes"], blocks=st["blocks_preempted"],
                              warps=st["warps_preempted"], done=st["warps_done"], step_ms=0.0, launches=2))
             del run
@@ -676,6 +689,18 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
     mode_id = {"ctxback": cb.MODE_CTXBACK, "full_hw": cb.MODE_FULL_HW, "none": cb.MODE_CTXBACK}
     results = {}
     refs = {}
+
+    def ls_alone_ms(n=10):
+        ts = []
+        for _ in range(n):
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            with torch.cuda.stream(hp):
+                a0.record(hp)
+                ls_job()
+                a1.record(hp)
+            hp.synchronize()
+            ts.append(a0.elapsed_time(a1))
+        return float(np.median(ts))
     for mode in modes:
         progs, grids, ctxs = {}, {}, {}
         for k, (txt, mb) in irs.items():
@@ -769,7 +794,8 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
                     ls_job()
                     hp.synchronize()
                     t_ls_done = time.perf_counter() - t0
-                    recs.append(dict(arr=t_arr, wait_ms=(t_ls_done - t_arr) * 1e3 - ls_ms,
+                    recs.append(dict(arr=t_arr, response_ms=(t_ls_done - t_arr) * 1e3,
+                                     wait_ms=(t_ls_done - t_arr) * 1e3 - ls_ms,
                                      host_to_ls_ms=(t_ls - t_arr) * 1e3, late_ms=(now - t_arr) * 1e3,
                                      preempt_call_ms=(tp1 - tp0) * 1e3, kind=job.kind,
                                      lat_us=st["latency_us"] if st and st["warps_preempted"] else None,
@@ -799,6 +825,7 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
 
         loop([], 0.3)                                           # warm-up
         base_recs, base_done, base_wall, bad0 = loop([], seconds / 2)
+        ls_ms = ls_alone_ms()                                   # isolated LS duration right before the trace
         arr = configs.c5_arrivals(seconds, 10.0, 51 + rank)
         recs, done, wall, bad = loop(arr, seconds)
         waits = np.array([r["wait_ms"] for r in recs]) if recs else np.zeros(1)
@@ -813,9 +840,11 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
             "latency_us_p50": float(np.median(lats)) if len(lats) else None,
             "latency_us_p99": float(np.percentile(lats, 99)) if len(lats) else None,
             "latency_us_max": float(lats.max()) if len(lats) else None,
+            "ls_response_ms_p50": float(np.median([r["response_ms"] for r in recs])) if recs else None,
+            "ls_alone_ms": ls_ms,
             "batch_jobs_per_s_no_arrivals": jobs_base, "batch_jobs_per_s_with_trace": jobs_trace,
             "ls_busy_fraction": busy,
-            "batch_throughput_loss_pct": 100.0 * (1 - jobs_trace / max(1e-9, jobs_base * (1 - busy))),
+            "batch_throughput_change_pct": 100.0 * (jobs_trace / max(1e-9, jobs_base) - 1.0),
             "jobs_done": done, "outputs_bit_exact": bad == 0 and bad0 == 0,
             "worst_arrivals": sorted(recs, key=lambda r: -r["wait_ms"])[:5],
         }
@@ -832,6 +861,8 @@ def gpu_arm(args):
     from workloads import configs
     ws, rank, local = dist_setup(args)
     torch.cuda.set_device(local)
+    clk = Clocks(local)
+    clk.start()
     size = args.size
     cfg = configs.c2(size, size, size)
     M = N = K = size
@@ -866,8 +897,6 @@ def gpu_arm(args):
     fr_t = rng.uniform(0.05, 0.95, args.steps)
     # ---- main timed loop: CTXBack ----
     preempt_steps(cb, pr, grid, (dA, dB, dC), ctxs["ctxback"], s, ctrl, ref, t_unint_ms / 1e3, fr_w, ws)
-    clk = Clocks(local)
-    clk.start()
     barrier(ws)
     torch.cuda.synchronize()
     recs = preempt_steps(cb, pr, grid, (dA, dB, dC), ctxs["ctxback"], s, ctrl, ref, t_unint_ms / 1e3, fr_t, ws)

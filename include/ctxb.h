@@ -131,6 +131,10 @@ typedef struct {
                                 warps (%globaltimer), "elapsed time before
                                 releasing the GPU"                                 */
   double host_us;            /* host: flag write issued -> victim stream drained   */
+  double signal_to_drained_us; /* CUDA events: event on ctrl right before the flag
+                                write -> the library's event after the victim
+                                kernel (every warp saved or done, kernel exited);
+                                negative if the kernel had finished already     */
   uint32_t warps_preempted, warps_done, blocks_preempted;
   uint64_t payload_bytes;    /* sum of saved payload over preempted warps          */
   uint64_t header_bytes;     /* 16 B per preempted warp                             */

@@ -61,7 +61,7 @@ struct ctxb_program {
   struct Res {
     CUdeviceptr flag = 0, stamps = 0, forced = 0;
     uint32_t n_warps = 0;
-    CUevent ev0 = nullptr, ev1 = nullptr;
+    CUevent ev0 = nullptr, ev1 = nullptr, evf = nullptr;
   };
   std::vector<Res> pool;   // per-run device resources, reused (flag is always left at 0)
   uint32_t full_ir_words128() const {  // 128-B rows occupied by the FULL_IR layout
@@ -98,10 +98,11 @@ struct ctxb_run {
   std::vector<uint32_t> hdr_prev, hdr;  // host header snapshots (launch e-1, e)
   bool resumed_launch = false;
   CUevent ev0 = nullptr, ev1 = nullptr;   // recorded around each launch on the run's stream
+  CUevent evf = nullptr;                  // recorded on the control stream before the flag write
   ~ctxb_run() {
     if (flag && prog) {   // return the resources to the program's pool
       std::lock_guard<std::mutex> g(prog->mu);
-      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1});
+      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf});
     }
   }
 };
@@ -336,6 +337,7 @@ int ctxb_program_destroy(ctxb_program* p) {
       d.cuMemFree(r.forced);
       d.cuEventDestroy(r.ev0);
       d.cuEventDestroy(r.ev1);
+      d.cuEventDestroy(r.evf);
     }
   }
   delete p;
@@ -474,6 +476,7 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
         r->forced = p->pool[i].forced;
         r->ev0 = p->pool[i].ev0;
         r->ev1 = p->pool[i].ev1;
+        r->evf = p->pool[i].evf;
         p->pool.erase(p->pool.begin() + (long)i);
         break;
       }
@@ -488,6 +491,7 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
     r->forced = t;
     CU(d.cuEventCreate(&r->ev0, CU_EVENT_DEFAULT));
     CU(d.cuEventCreate(&r->ev1, CU_EVENT_DEFAULT));
+    CU(d.cuEventCreate(&r->evf, CU_EVENT_DEFAULT));
     std::vector<uint32_t> z(64, 0);
     CU(d.cuMemcpyHtoD(r->flag, z.data(), 256));   // the flag is 0 whenever a run does not hold it raised
   }
@@ -509,6 +513,7 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     return fail(CTXB_E_INVALID_ARG, "ctrl_stream must differ from the run's stream");
   Driver& d = driver();
   double t0 = now_ms();
+  CU(d.cuEventRecord(r->evf, (CUstream)ctrl));
   CU(d.cuStreamWriteValue32((CUstream)ctrl, r->flag, 1u, 0));
   CU(d.cuStreamSynchronize(r->stream));
   double t1 = now_ms();
@@ -539,6 +544,10 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     }
     for (auto b : blk) st->blocks_preempted += b;
     st->latency_us = st->warps_preempted ? (double)(tmax - tmin) * 1e-3 : 0.0;
+    CU(d.cuStreamSynchronize((CUstream)ctrl));
+    float ms = 0;
+    CU(d.cuEventElapsedTime(&ms, r->evf, r->ev1));
+    st->signal_to_drained_us = (double)ms * 1e3;
   }
   return CTXB_OK;
 }

@@ -66,7 +66,8 @@ class _ProgInfo(C.Structure):
 
 
 class _PreStats(C.Structure):
-    _fields_ = [("latency_us", C.c_double), ("host_us", C.c_double), ("warps_preempted", C.c_uint32),
+    _fields_ = [("latency_us", C.c_double), ("host_us", C.c_double), ("signal_to_drained_us", C.c_double),
+                ("warps_preempted", C.c_uint32),
                 ("warps_done", C.c_uint32), ("blocks_preempted", C.c_uint32), ("payload_bytes", C.c_uint64),
                 ("header_bytes", C.c_uint64)]
 
