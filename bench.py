@@ -379,13 +379,14 @@ def oracle_sample(steps=1, seed=0):
 
 # ---- the other BASELINE configs (configs[0], [2], [3]) ----------------------
 
-MODES = (("ctxback", 0), ("full_hw", 3), ("live", 1))
+MODES = (("ctxback", 0, 7), ("full_hw", 3, 7), ("live", 1, 7),
+         ("cs_defer", 1, 15), ("ctxback_cs_defer", 0, 15))      # (name, mode, flags); 15 = ALL | DEFER
 
 
 def _progs(cb, ir_text, debug=0, min_blocks=0):
     return {name: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT if "poll" in ir_text else cb.POLL_EVERY_INSTR,
-                             mode=mode, debug=debug, min_blocks_per_sm=min_blocks)
-            for name, mode in MODES}
+                             mode=mode, flags=flags, debug=debug, min_blocks_per_sm=min_blocks)
+            for name, mode, flags in MODES}
 
 
 def _grid(progs):
@@ -436,8 +437,9 @@ def _flag_trials(progs, grid, make_bufs, uniforms, check, fracs, T_s):
     return out
 
 
-def _reduction(res):
-    c, f = res.get("ctxback", {}), res.get("full_hw", {})
+def _reduction(res, name="ctxback"):
+    c, f = res.get(name, {}), res.get("full_hw", {})
+
     def pct(k):
         if c.get(k) and f.get(k):
             return round(100 * (1 - c[k] / f[k]), 2)
@@ -454,8 +456,8 @@ def bench_c1(cb):
     cfg = configs.c1()
     names = ["in0", "in1", "rw0", "out"]
     res = {}
-    for name, mode in MODES:
-        prog = cb.Program(cfg["ir"], mode=mode, debug=cb.DEBUG_FORCED)
+    for name, mode, flags in MODES:
+        prog = cb.Program(cfg["ir"], mode=mode, flags=flags, debug=cb.DEBUG_FORCED)
         ctx = torch.zeros(prog.context_capacity(1), dtype=torch.uint8, device="cuda")
         dev = {n: torch.from_numpy(cfg["buffers"][n].view(np.int32).copy()).cuda() for n in names}
         ref = None
@@ -485,6 +487,8 @@ def bench_c1(cb):
         if name == "ctxback":
             res["static"] = _static(prog, 4)
     res["reduction_vs_full_hw"] = _reduction(res)
+    res["cs_defer_reduction_vs_full_hw"] = _reduction(res, "cs_defer")
+    res["ctxback_cs_defer_reduction_vs_full_hw"] = _reduction(res, "ctxback_cs_defer")
     res["workload"] = "C1 24-instruction IR kernel, 1 TB x 128 threads, all warps preempted at each of the 24 sites"
     return res
 
@@ -513,6 +517,8 @@ def bench_c3(cb, trials, seed):
     res = _flag_trials(progs, grid, make, [], lambda b: bool(torch.equal(b[1], ref)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
     res["reduction_vs_full_hw"] = _reduction(res)
+    res["cs_defer_reduction_vs_full_hw"] = _reduction(res, "cs_defer")
+    res["ctxback_cs_defer_reduction_vs_full_hw"] = _reduction(res, "ctxback_cs_defer")
     res["t_uninterrupted_ms"] = round(T, 3)
     res["grid"] = grid
     res["uninterrupted_equals_numpy"] = ok

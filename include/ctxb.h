@@ -60,6 +60,11 @@ extern "C" {
 #define CTXB_REVERT   2u  /* instruction reverting, Alg. 2            */
 #define CTXB_OSRB     4u  /* on-chip scalar register backup           */
 #define CTXB_ALL      7u
+#define CTXB_DEFER    8u  /* CS-Defer (ref [4]): a preemption arriving at a
+                             site may continue to a later site of the same basic
+                             block whose estimated latency is lower; combined
+                             with CTXBack plans = CTXBack+CS-Defer,
+                             with CTXB_MODE_LIVE = CS-Defer                       */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */
@@ -95,6 +100,9 @@ typedef struct {
   uint32_t min_blocks_per_sm; /* 0 = compiler's choice; else both generated kernels
                            get __launch_bounds__(block, n): ptxas caps registers
                            so n blocks fit per SM (persistent-grid occupancy)      */
+  uint32_t defer_instr_bytes; /* CTXB_DEFER latency estimate: one deferred instruction
+                           costs this many context bytes (0 = 8); the stalls of the
+                           deferred instructions are ignored, as in P:380          */
 } ctxb_options;
 
 typedef struct ctxb_program ctxb_program; /* analysed IR kernel + module; library-owned */
@@ -111,6 +119,8 @@ typedef struct {
   uint32_t n_reexec;        /* re-executed instructions at resume (Alg. 1)          */
   uint32_t payload_bytes_per_warp; /* 128*n_vec + 4*n_scalar                        */
   uint32_t live_bytes_per_warp;    /* the LIVE plan of the same site (fallback)     */
+  uint32_t defer_site;             /* CTXB_DEFER: site a preemption arriving here is
+                                      carried to (== this site: no deferral)          */
 } ctxb_site_info_t;
 
 typedef struct {
@@ -150,7 +160,7 @@ const char* ctxb_version(void);
 
 /* Parse + analyse + generate + compile.  `ir_text` need not be
  * NUL-terminated (`len` bytes are read).  opts == NULL means
- * {CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0}.
+ * {CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8}.
  * Errors: _INVALID_ARG, _PARSE, _ANALYSIS, _NVRTC. */
 int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb_program** out);
 int ctxb_program_destroy(ctxb_program* prog);

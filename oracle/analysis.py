@@ -42,6 +42,9 @@ FLAG_RELAXED = 1
 FLAG_REVERT = 2
 FLAG_OSRB = 4
 FLAGS_ALL = 7
+FLAG_DEFER = 8            # CS-Defer on top of the mode's own plans
+
+DEFER_INSTR_BYTES = 8     # latency-estimate weight of one deferred instruction, in context bytes
 
 MODE_CTXBACK = 0
 MODE_LIVE = 1
@@ -530,6 +533,7 @@ class Analysis:
     candidates: dict = field(default_factory=dict)   # c -> {p: Plan or None}
     mode: int = MODE_CTXBACK
     flags: int = FLAGS_ALL
+    defer: dict = field(default_factory=dict)        # site c -> site it defers to (c itself: none)
 
 
 def best_plan(prog, lv, heads, c, backups, flags, keep=None):
@@ -570,9 +574,41 @@ def osrb_candidates(prog):
     return out
 
 
+def defer_targets(prog, sites, plans, instr_bytes=DEFER_INSTR_BYTES):
+    """CS-Defer and its combination with the site's own plan
+    (P:325-329): a preemption arriving at site c may continue to a later site
+    d of the same basic block (control flow must stay determinable) and
+    save d's context there.  The paper ranks the options by estimated
+    preemption latency and ignores the stalls of the in-between instructions
+    (P:380); here E(c -> d) = bytes(plan at d) + instr_bytes * (d - c), and d
+    minimises E over d >= c (ties: the earliest d, i.e. no deferral first)."""
+    out = {}
+    for c in sites:
+        bb = prog.bb_of(c)
+        best, best_e = c, None
+        for d in sites:
+            if d < c or prog.bb_of(d) != bb:
+                continue
+            e = plans[d].payload_bytes + instr_bytes * (d - c)
+            if best_e is None or e < best_e:
+                best, best_e = d, e
+        out[c] = best
+    return out
+
+
 def analyze(prog: Program, policy="EVERY_INSTR", mode=MODE_CTXBACK, flags=FLAGS_ALL,
-            every=8, sites=None, keep_candidates=False) -> Analysis:
+            every=8, sites=None, keep_candidates=False, defer_instr_bytes=DEFER_INSTR_BYTES) -> Analysis:
     """Compile-time analysis: per poll site, the chosen plan."""
+    an = _analyze(prog, policy, mode, flags & FLAGS_ALL, every, sites, keep_candidates)
+    an.flags = flags
+    if flags & FLAG_DEFER:
+        an.defer = defer_targets(prog, an.sites, an.plans, defer_instr_bytes)
+    else:
+        an.defer = {c: c for c in an.sites}
+    return an
+
+
+def _analyze(prog, policy, mode, flags, every, sites, keep_candidates):
     lv = liveness(prog)
     heads = region_heads(prog)
     if sites is None:

@@ -208,6 +208,10 @@ class Machine:
         self.status = np.zeros(self.nW, dtype=np.int8)   # 0 run, 1 parked, 2 done
         self.parked = {}           # local warp -> (c, plan, ctx)
         self.resumed_pass = np.zeros(self.nW, dtype=bool)
+        # CS-Defer: a preemption decided at site c is carried to the
+        # site it defers to; pend[w] = that site + 1 (0 = nothing pending)
+        self.pend = np.zeros(self.nW, dtype=np.int64)
+        self.defer = dict(an.defer) if an.defer else {c: c for c in an.sites}
 
     # --- operand access ----------------------------------------------------------
     def _opd(self, o, g):
@@ -426,6 +430,7 @@ class Machine:
                 self.S[int(r[1:])][w] = _u(x).reshape(-1)[0]
         self.status[w] = 0
         self.resumed_pass[w] = True
+        self.pend[w] = 0
         return c
 
     def _final_value(self, plan, r):
@@ -496,10 +501,19 @@ class Machine:
                     if len(pw):
                         hit = count[pw] == targets[pw]
                         count[pw] += 1
-                        if np.any(hit):
-                            for w in pw[hit]:
+                        pend = self.pend[pw]
+                        save = (pend == pc + 1)                      # a deferred preemption lands here
+                        start = (pend == 0) & hit
+                        d = self.defer.get(pc, pc)
+                        if d != pc:
+                            self.pend[pw[start]] = d + 1             # continue to the deferral target
+                        else:
+                            save = save | start
+                        self.pend[pw[save]] = 0
+                        if np.any(save):
+                            for w in pw[save]:
                                 self._preempt(int(w), pc)
-                            g = g[~np.isin(g, pw[hit])]
+                            g = g[~np.isin(g, pw[save])]
                             if not len(g):
                                 break
                 outs = self._exec(pc, g)

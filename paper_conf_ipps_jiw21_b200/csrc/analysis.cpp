@@ -19,7 +19,7 @@
 namespace ctxb {
 namespace {
 
-constexpr uint32_t F_RELAXED = 1, F_REVERT = 2, F_OSRB = 4;
+constexpr uint32_t F_RELAXED = 1, F_REVERT = 2, F_OSRB = 4, F_DEFER = 8;
 constexpr uint32_t VEC_B = 128, SCA_B = 4;
 
 bool is_alu(Op o) {
@@ -567,7 +567,48 @@ std::vector<int> Plan::cost() const {
   return {(int)payload_bytes, (int)n_rev_pre, (int)(n_reexec + n_rev_res), -p};
 }
 
+// CS-Defer combined with the site's own plans: a
+// preemption arriving at site k may continue to a later site k' of the same
+// basic block and save there.  Estimated latency (stalls of the in-between
+// instructions ignored, as in the paper):
+//   E(k -> k') = bytes(plan at k') + defer_instr_bytes * (c_k' - c_k),
+// k' minimises E (ties: the earliest k', i.e. no deferral first).
+static std::vector<int> defer_targets(const Program& P, const Analysis& A, uint32_t instr_bytes) {
+  std::vector<int> out(A.sites.size());
+  for (size_t k = 0; k < A.sites.size(); k++) {
+    int c = A.sites[k], bb = P.bb_of[c];
+    size_t best = k;
+    uint64_t best_e = UINT64_MAX;
+    for (size_t q = 0; q < A.sites.size(); q++) {
+      int d = A.sites[q];
+      if (d < c || P.bb_of[d] != bb) continue;
+      uint64_t e = (uint64_t)A.plans[q].payload_bytes + (uint64_t)instr_bytes * (uint64_t)(d - c);
+      if (e < best_e) {
+        best_e = e;
+        best = q;
+      }
+    }
+    out[k] = (int)best;
+  }
+  return out;
+}
+
+static Analysis analyze_plans(const Program& P, const Options& opt);
+
 Analysis analyze(const Program& P, const Options& opt) {
+  Analysis A = analyze_plans(P, opt);
+  if (opt.flags & F_DEFER) {
+    A.defer = defer_targets(P, A, opt.defer_instr_bytes);
+  } else {
+    A.defer.resize(A.sites.size());
+    for (size_t k = 0; k < A.sites.size(); k++) A.defer[k] = (int)k;
+  }
+  return A;
+}
+
+static Analysis analyze_plans(const Program& P, const Options& opt0) {
+  Options opt = opt0;
+  opt.flags &= 7u;
   Liveness L = liveness(P);
   DefIndex D(P);
   Analysis A;

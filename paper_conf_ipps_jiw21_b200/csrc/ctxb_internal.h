@@ -138,6 +138,7 @@ struct Plan {
 
 struct Options {
   uint32_t flags = 7, mode = 0, policy = 0, every = 8, debug = 0, flag_depth = 1, min_blocks = 0;
+  uint32_t defer_instr_bytes = 8;   // CS-Defer latency-estimate weight per deferred instruction
 };
 
 struct Analysis {
@@ -147,6 +148,7 @@ struct Analysis {
   std::vector<int> backups;                             // OSRB-selected instructions
   std::vector<Plan> plans;                              // per site (index into sites)
   std::vector<Plan> live;                               // LIVE plan per site
+  std::vector<int> defer;                               // per site: index of the site it defers to
   uint32_t full_ir_bytes = 0;
 };
 

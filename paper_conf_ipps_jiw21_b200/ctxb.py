@@ -14,7 +14,7 @@ import numpy as np
 
 __all__ = [
     "LIB_PATH", "CtxbError", "lib",
-    "RELAXED", "REVERT", "OSRB", "ALL", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
+    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
     "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "EXPORTED_SYMBOLS",
@@ -25,7 +25,7 @@ __all__ = [
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libctxb.so")
 
-RELAXED, REVERT, OSRB, ALL = 1, 2, 4, 7
+RELAXED, REVERT, OSRB, ALL, DEFER = 1, 2, 4, 7, 8
 MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
 DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE = 1, 2, 4, 8
@@ -50,12 +50,13 @@ class CtxbError(RuntimeError):
 class _Opts(C.Structure):
     _fields_ = [("flags", C.c_uint32), ("mode", C.c_uint32), ("poll_policy", C.c_uint32),
                 ("poll_every", C.c_uint32), ("debug", C.c_uint32), ("flag_depth", C.c_uint32),
-                ("min_blocks_per_sm", C.c_uint32)]
+                ("min_blocks_per_sm", C.c_uint32), ("defer_instr_bytes", C.c_uint32)]
 
 
 class _SiteInfo(C.Structure):
     _fields_ = [(n, C.c_uint32) for n in ("c", "p", "n_vec", "n_scalar", "n_revert_pre", "n_revert_res",
-                                          "n_reexec", "payload_bytes_per_warp", "live_bytes_per_warp")]
+                                          "n_reexec", "payload_bytes_per_warp", "live_bytes_per_warp",
+                                          "defer_site")]
 
 
 class _ProgInfo(C.Structure):
@@ -149,8 +150,9 @@ def _u32arr(vals):
 # --- the C-ABI names ----------------------------------------------------------
 
 def ctxb_analyze(ir_text: str, flags=ALL, mode=MODE_CTXBACK, poll_policy=POLL_EVERY_INSTR, poll_every=8,
-                 debug=0, flag_depth=1, min_blocks_per_sm=0) -> "Program":
-    return Program(ir_text, flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm)
+                 debug=0, flag_depth=1, min_blocks_per_sm=0, defer_instr_bytes=8) -> "Program":
+    return Program(ir_text, flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm,
+                   defer_instr_bytes)
 
 
 def ctxb_launch(prog, grid, buffers, uniforms, ctx, stream=None, forced=None) -> "Run":
@@ -185,9 +187,9 @@ class Program:
     """An analysed + compiled IR kernel (ctxb_analyze)."""
 
     def __init__(self, ir_text, flags=ALL, mode=MODE_CTXBACK, poll_policy=POLL_EVERY_INSTR, poll_every=8,
-                 debug=0, flag_depth=1, min_blocks_per_sm=0):
+                 debug=0, flag_depth=1, min_blocks_per_sm=0, defer_instr_bytes=8):
         self._h = C.c_void_p()
-        o = _Opts(flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm)
+        o = _Opts(flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm, defer_instr_bytes)
         b = ir_text.encode()
         _chk(lib.ctxb_analyze(b, len(b), C.byref(o), C.byref(self._h)))
         self.debug = debug

@@ -27,13 +27,14 @@ def _cb():
     return cb
 
 
-def check(txt, grid, bufs, schedules, policy="EVERY_INSTR", skip=("scr",), poison=True, flags=7):
+def check(txt, grid, bufs, schedules, policy="EVERY_INSTR", skip=("scr",), poison=True, flags=7, mode=0,
+          defer_instr_bytes=8):
     cb = _cb()
     op = ir.parse(txt)
-    an = A.analyze(op, policy=policy, flags=flags)
+    an = A.analyze(op, policy=policy, flags=flags, mode=mode, defer_instr_bytes=defer_instr_bytes)
     pol = {"EVERY_INSTR": cb.POLL_EVERY_INSTR, "EXPLICIT": cb.POLL_EXPLICIT}[policy]
     dbg = cb.DEBUG_FORCED | (cb.DEBUG_POISON if poison else 0)
-    prog = cb.Program(txt, flags=flags, poll_policy=pol, debug=dbg)
+    prog = cb.Program(txt, flags=flags, poll_policy=pol, debug=dbg, mode=mode, defer_instr_bytes=defer_instr_bytes)
     names = list(op.buffers)
     ref, _ = interp.run(an, grid, bufs)
     g0, h0, _ = gpu_run(prog, names, grid, bufs, {})
@@ -110,3 +111,27 @@ def test_paper_figures_on_gpu(name):
             for b, k in op.buffers.items()}
     n = len(op.instrs)
     check(g["ir"], 1, bufs, [[[k]] for k in range(n)])
+
+
+@pytest.mark.parametrize("mode", [0, 1])
+def test_c1_cs_defer(mode):
+    """CS-Defer (mode LIVE + DEFER) and CTXBack+CS-Defer (CTXBACK + DEFER):
+    preemptions carried to their deferral target, bit-exact, bytes = oracle."""
+    cfg = configs.c1()
+    vecs = configs.c1_random_site_vectors(64, seed=9)
+    scheds = [[[k] * 4] for k in range(24)] + [[v] for v in vecs]
+    check(cfg["ir"], 1, cfg["buffers"], scheds, flags=15, mode=mode)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_random_programs_defer(seed):
+    loop = seed % 3 == 0
+    txt, size = random_program(400 + seed, loop=loop, n_body=10)
+    op = ir.parse(txt)
+    grid = 2
+    nout = op.nv - 1 + op.ns - (1 if loop else 0)
+    bufs = random_buffers(seed, op.block, grid, size, nout)
+    r = np.random.default_rng(seed)
+    nw = grid * op.nwarps
+    scheds = [[r.integers(0, 60, nw).astype(np.uint32), r.integers(0, 20, nw).astype(np.uint32)] for _ in range(4)]
+    check(txt, grid, bufs, scheds, flags=15, mode=seed % 2, defer_instr_bytes=2)
