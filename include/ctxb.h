@@ -86,6 +86,8 @@ extern "C" {
 #define CTXB_DEBUG_NO_POLLS   4u /* compile poll sites out (overhead baseline;
                                     the kernel cannot be preempted)            */
 #define CTXB_DEBUG_NO_COMPILE 8u /* analysis + code generation only            */
+#define CTXB_DEBUG_NO_SHARE  16u /* one preemption routine per site (no P:317
+                                    sharing of identical routines)             */
 
 typedef struct {
   uint32_t flags;       /* CTXB_RELAXED | CTXB_REVERT | CTXB_OSRB                */
@@ -133,6 +135,9 @@ typedef struct {
   uint32_t resume_maxnreg;             /* min blocks/SM requested for the resume kernel
                                           (__launch_bounds__) so it keeps the normal
                                           kernel's occupancy (0 = none needed)       */
+  uint32_t n_save_stubs;               /* distinct preemption-routine bodies after
+                                          sharing                            */
+  uint32_t cubin_bytes;                /* size of the compiled sm_100a cubin         */
   double analyze_ms, codegen_ms, compile_ms;
 } ctxb_program_info_t;
 

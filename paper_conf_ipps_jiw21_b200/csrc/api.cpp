@@ -200,7 +200,9 @@ int compile(ctxb_program* p) {
   if (bs < bw && bw > 0) {
     // ask ptxas for the normal kernel's occupancy (__launch_bounds__ min blocks)
     p->cg.resume_maxnreg = bw;
+    uint32_t nss = p->cg.n_save_stubs;
     p->src = generate_cuda(p->prog, p->an, p->opt, &p->cg);
+    (void)nss;
     rc = nvrtc_compile(p, &rr, &rs);
     if (rc) return rc;
   }
@@ -361,6 +363,8 @@ int ctxb_program_info(const ctxb_program* p, ctxb_program_info_t* o) {
   o->compiled = p->cubin.empty() ? 0 : 1;
   o->num_regs_resume = p->regs_resume;
   o->resume_maxnreg = p->cg.resume_maxnreg;
+  o->n_save_stubs = p->cg.n_save_stubs;
+  o->cubin_bytes = (uint32_t)p->cubin.size();
   o->analyze_ms = p->t_an;
   o->codegen_ms = p->t_cg;
   o->compile_ms = p->t_cc;

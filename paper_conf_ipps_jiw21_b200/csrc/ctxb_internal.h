@@ -160,6 +160,7 @@ struct CodegenInfo {
   uint32_t stride = 0;            // payload slot bytes per warp (multiple of 128)
   uint32_t max_payload = 0;
   uint32_t resume_maxnreg = 0;    // in: register cap of the resume kernel (0 = none)
+  uint32_t n_save_stubs = 0;      // out: distinct preemption-routine bodies (P:317 sharing)
 };
 std::string generate_cuda(const Program& prog, const Analysis& an, const Options& opt,
                           CodegenInfo* info);

@@ -16,7 +16,7 @@ __all__ = [
     "LIB_PATH", "CtxbError", "lib",
     "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
-    "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE",
+    "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "EXPORTED_SYMBOLS",
     "ctxb_analyze", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait", "ctxb_context_bytes",
     "ctxb_flag_propagation",
@@ -28,7 +28,7 @@ LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libctxb.so"
 RELAXED, REVERT, OSRB, ALL, DEFER = 1, 2, 4, 7, 8
 MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
-DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE = 1, 2, 4, 8
+DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1, 2, 4, 8, 16
 STATE_NONE, STATE_PREEMPTED, STATE_DONE = 0, 1, 2
 NEVER = 0xFFFFFFFF
 
@@ -62,7 +62,8 @@ class _SiteInfo(C.Structure):
 class _ProgInfo(C.Structure):
     _fields_ = [(n, C.c_uint32) for n in ("n_instrs", "nv", "ns", "block", "n_buffers", "n_uniforms", "n_sites",
                                           "n_backups", "max_payload_bytes_per_warp", "full_ir_bytes_per_warp",
-                                          "num_regs", "compiled", "num_regs_resume", "resume_maxnreg")] + \
+                                          "num_regs", "compiled", "num_regs_resume", "resume_maxnreg",
+                                          "n_save_stubs", "cubin_bytes")] + \
                [("analyze_ms", C.c_double), ("codegen_ms", C.c_double), ("compile_ms", C.c_double)]
 
 
