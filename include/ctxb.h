@@ -65,6 +65,10 @@ extern "C" {
                              block whose estimated latency is lower; combined
                              with CTXBack plans = CTXBack+CS-Defer,
                              with CTXB_MODE_LIVE = CS-Defer                       */
+#define CTXB_PRUNE   16u  /* demand-driven restore (NEXT N4): restore only what the
+                             registers live at the site need, instead of every
+                             live-out result of the window (R-2, literal); every
+                             flashback-point becomes feasible                     */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */

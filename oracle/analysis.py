@@ -43,6 +43,7 @@ FLAG_REVERT = 2
 FLAG_OSRB = 4
 FLAGS_ALL = 7
 FLAG_DEFER = 8            # CS-Defer on top of the mode's own plans
+FLAG_PRUNE = 16           # demand-driven restore (NEXT N4): restore only what LIVE_IN(c) needs
 
 DEFER_INSTR_BYTES = 8     # latency-estimate weight of one deferred instruction, in context bytes
 
@@ -372,7 +373,16 @@ class _Window:
     # --- context accounting (R-6, R-8) ---
 
     def demands(self):
-        """Resume-time demands: (value, supply) pairs."""
+        """Resume-time demands: (value, supply) pairs.  R-2 (literal): every
+        re-executable instruction's operands and every live-out result of the
+        window.  FLAG_PRUNE: only the final value of each register live-in at
+        I_cur; re-executions are then demanded transitively (compute_S)."""
+        if self.flags & FLAG_PRUNE:
+            out = []
+            for r in sorted(self.lv.live_in[self.c]):
+                d = self.rd(r, self.c)
+                out.append(((r, d), self.supply_of((r, d)) if d is not PRE else ("C",)))
+            return out
         out = []
         for j in self.W:
             if j in self.reexec:
@@ -387,9 +397,12 @@ class _Window:
         return out
 
     def compute_S(self, pos):
-        """Saved set S, reverts run at resume, reverts run at preempt."""
+        """Saved set S, reverts run at resume, reverts run at preempt (and,
+        with FLAG_PRUNE, the re-executions the demands reach)."""
         S = {}
         used_res, used_pre = set(), set()
+        used_x = set()
+        prune = bool(self.flags & FLAG_PRUNE)
 
         def pre_closure(v):
             if v in used_pre:
@@ -407,7 +420,11 @@ class _Window:
             elif k == "B":
                 S.setdefault(v, "B")
             elif k == "X":
-                pass
+                j = s[1]
+                if prune and j not in used_x:
+                    used_x.add(j)
+                    for x, sx in zip(self.opvals(j), self.reexec[j]):
+                        demand(x, sx)
             elif k == "R":
                 if pos.get(v, "R") == "P":
                     S.setdefault(v, "P")
@@ -421,6 +438,7 @@ class _Window:
                         demand(x, sx)
         for v, s in self.demands():
             demand(v, s)
+        self._used_x = used_x if prune else set(self.reexec)
         return S, used_res, used_pre
 
     def plan(self, kind="ctxback"):
@@ -439,11 +457,12 @@ class _Window:
             if bP < bR:
                 pos[v] = "P"
         S, used_res, used_pre = self.compute_S(pos)
+        used_x = self._used_x
         saved = sorted(((src, v) for v, src in S.items()), key=_saved_key)
         pre_list = sorted(used_pre, key=lambda x: -self.rev[x][0])
         preempt_reverts = [(v,) + tuple(self.rev[v]) for v in pre_list]
         schedule = [e for e in self.events
-                    if e[0] == "X" or (e[0] == "R" and e[1] in used_res)]
+                    if (e[0] == "X" and e[1] in used_x) or (e[0] == "R" and e[1] in used_res)]
         final = {}
         for r in sorted(self.lv.live_in[self.c]):
             d = self.rd(r, self.c)
@@ -452,8 +471,8 @@ class _Window:
         nv = sum(1 for v in S if prog.is_vector(v[0]))
         bkp = {v: d[1] for v, d in self.valid.items() if d[0] == "B"}
         return Plan(self.c, self.p, kind, saved, preempt_reverts, schedule,
-                    dict(self.reexec), dict(self.rev), final, nb, nv, len(S) - nv,
-                    len(used_pre), len(used_res), len(self.reexec), bkp)
+                    {j: self.reexec[j] for j in used_x}, dict(self.rev), final, nb, nv, len(S) - nv,
+                    len(used_pre), len(used_res), len(used_x), bkp)
 
 
 def _saved_key(item):
@@ -468,7 +487,7 @@ def plan_window(prog, lv, p, c, backups=(), flags=FLAGS_ALL):
         return basic_plan(prog, lv, p, c)
     w = _Window(prog, lv, p, c, set(backups) if (flags & FLAG_OSRB) else set(), flags)
     w.sweep()
-    if not w.feasible():
+    if not (flags & FLAG_PRUNE) and not w.feasible():
         return None
     return w.plan()
 
@@ -599,7 +618,7 @@ def defer_targets(prog, sites, plans, instr_bytes=DEFER_INSTR_BYTES):
 def analyze(prog: Program, policy="EVERY_INSTR", mode=MODE_CTXBACK, flags=FLAGS_ALL,
             every=8, sites=None, keep_candidates=False, defer_instr_bytes=DEFER_INSTR_BYTES) -> Analysis:
     """Compile-time analysis: per poll site, the chosen plan."""
-    an = _analyze(prog, policy, mode, flags & FLAGS_ALL, every, sites, keep_candidates)
+    an = _analyze(prog, policy, mode, flags & (FLAGS_ALL | FLAG_PRUNE), every, sites, keep_candidates)
     an.flags = flags
     if flags & FLAG_DEFER:
         an.defer = defer_targets(prog, an.sites, an.plans, defer_instr_bytes)

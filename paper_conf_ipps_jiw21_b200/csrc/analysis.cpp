@@ -19,7 +19,7 @@
 namespace ctxb {
 namespace {
 
-constexpr uint32_t F_RELAXED = 1, F_REVERT = 2, F_OSRB = 4, F_DEFER = 8;
+constexpr uint32_t F_RELAXED = 1, F_REVERT = 2, F_OSRB = 4, F_DEFER = 8, F_PRUNE = 16;
 constexpr uint32_t VEC_B = 128, SCA_B = 4;
 
 bool is_alu(Op o) {
@@ -326,8 +326,20 @@ class Window {
     return true;
   }
 
+  // Resume-time demands.  R-2 (literal): every re-executed instruction's
+  // operands and every live-out result of the window.  F_PRUNE (demand-driven
+  // restore): only the final value of each register live-in at I_cur;
+  // re-executions are then demanded transitively in compute_S.
   std::vector<std::pair<Val, Supply>> demands() const {
     std::vector<std::pair<Val, Supply>> out;
+    if (flags & F_PRUNE) {
+      for (int r = 0; r < P.nregs(); r++)
+        if (L.in[c][r]) {
+          int d = rd(r, c);
+          out.push_back({{r, d}, d == PRE ? Supply{SK::C, -1} : supply_of({r, d})});
+        }
+      return out;
+    }
     for (int j = p; j < c; j++)
       if (reexec[j - p]) {
         auto ov = opvals(j);
@@ -347,6 +359,7 @@ class Window {
   struct SRes {
     std::map<Val, char> S;
     std::set<Val> used_res, used_pre;
+    std::set<int> used_x;   // re-executions the demands reach (all of them without F_PRUNE)
   };
 
   SRes compute_S(const std::map<Val, char>& pos) const {
@@ -362,7 +375,14 @@ class Window {
       switch (s.k) {
         case SK::C: R.S.emplace(v, 'C'); break;
         case SK::B: R.S.emplace(v, 'B'); break;
-        case SK::X: break;
+        case SK::X:
+          if ((flags & F_PRUNE) && !R.used_x.count(s.arg)) {
+            R.used_x.insert(s.arg);
+            auto ov = opvals(s.arg);
+            const auto& sup = rx_supply.at(s.arg);
+            for (size_t k = 0; k < ov.size(); k++) demand(ov[k], sup[k]);
+          }
+          break;
         case SK::R: {
           auto it = pos.find(v);
           char ps = it == pos.end() ? 'R' : it->second;
@@ -380,6 +400,9 @@ class Window {
       }
     };
     for (auto& [v, s] : demands()) demand(v, s);
+    if (!(flags & F_PRUNE))
+      for (int j = p; j < c; j++)
+        if (reexec[j - p]) R.used_x.insert(j);
     return R;
   }
 
@@ -430,8 +453,8 @@ class Window {
     std::stable_sort(pre.begin(), pre.end(), [&](const Val& a, const Val& b) { return revs.at(a).m > revs.at(b).m; });
     for (auto& v : pre) pl.pre_reverts.push_back(revs.at(v));
     for (auto& e : events)
-      if (e.is_x || fin.used_res.count(e.v)) pl.schedule.push_back(e);
-    pl.reexec_supply = rx_supply;
+      if ((e.is_x && fin.used_x.count(e.j)) || (!e.is_x && fin.used_res.count(e.v))) pl.schedule.push_back(e);
+    for (int j : fin.used_x) pl.reexec_supply[j] = rx_supply.at(j);
     pl.revert_info = revs;
     for (int r = 0; r < P.nregs(); r++)
       if (L.in[c][r]) {
@@ -442,9 +465,7 @@ class Window {
     for (auto& [v, src] : fin.S) (P.is_vec(v.r) ? pl.n_vec : pl.n_sca)++;
     pl.n_rev_pre = (uint32_t)fin.used_pre.size();
     pl.n_rev_res = (uint32_t)fin.used_res.size();
-    uint32_t nx = 0;
-    for (auto x : reexec) nx += x;
-    pl.n_reexec = nx;
+    pl.n_reexec = (uint32_t)fin.used_x.size();
     return pl;
   }
 
@@ -504,7 +525,7 @@ Plan window_plan(const Program& P, const Liveness& L, const DefIndex& D, int p, 
   if (!(flags & F_RELAXED)) return basic_plan(P, L, D, p, c);
   Window w(P, L, D, p, c, (flags & F_OSRB) ? bk : std::vector<int>{}, flags);
   w.sweep();
-  if (!w.feasible()) return Plan{};
+  if (!(flags & F_PRUNE) && !w.feasible()) return Plan{};
   return w.plan(0);
 }
 
@@ -608,7 +629,7 @@ Analysis analyze(const Program& P, const Options& opt) {
 
 static Analysis analyze_plans(const Program& P, const Options& opt0) {
   Options opt = opt0;
-  opt.flags &= 7u;
+  opt.flags &= (7u | F_PRUNE);
   Liveness L = liveness(P);
   DefIndex D(P);
   Analysis A;

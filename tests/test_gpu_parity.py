@@ -135,3 +135,25 @@ def test_random_programs_defer(seed):
     nw = grid * op.nwarps
     scheds = [[r.integers(0, 60, nw).astype(np.uint32), r.integers(0, 20, nw).astype(np.uint32)] for _ in range(4)]
     check(txt, grid, bufs, scheds, flags=15, mode=seed % 2, defer_instr_bytes=2)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_random_programs_prune(seed):
+    """Demand-driven restore (CTXB_PRUNE, NEXT N4) on the GPU vs the oracle."""
+    loop = seed % 3 == 0
+    txt, size = random_program(500 + seed, loop=loop, n_body=10)
+    op = ir.parse(txt)
+    grid = 2
+    nout = op.nv - 1 + op.ns - (1 if loop else 0)
+    bufs = random_buffers(seed, op.block, grid, size, nout)
+    r = np.random.default_rng(seed)
+    nw = grid * op.nwarps
+    scheds = [[r.integers(0, 60, nw).astype(np.uint32), r.integers(0, 20, nw).astype(np.uint32)] for _ in range(4)]
+    check(txt, grid, bufs, scheds, flags=23)
+
+
+def test_c2_half_prune_small():
+    cfg = configs.c2(128, 128, 32, polls="half")
+    r = np.random.default_rng(2)
+    scheds = [[r.integers(0, 64, 8).astype(np.uint32), r.integers(0, 8, 8).astype(np.uint32)] for _ in range(3)]
+    check(cfg["ir"], 1, cfg["buffers"], scheds, policy="EXPLICIT", flags=23)
