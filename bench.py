@@ -50,7 +50,7 @@ def parse():
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-oracle", action="store_true")
     ap.add_argument("--seed", type=int, default=100)
-    ap.add_argument("--configs", default="c1,c3,c4a,c4b,c5",
+    ap.add_argument("--configs", default="c1,c2s,c3,c4a,c4b,c5",
                     help="extra BASELINE configs measured after the C2 headline (comma list, or 'none')")
     ap.add_argument("--config-trials", type=int, default=5)
     ap.add_argument("--c5-seconds", type=float, default=4.0)
@@ -490,6 +490,40 @@ def bench_c1(cb):
     res["cs_defer_reduction_vs_full_hw"] = _reduction(res, "cs_defer")
     res["ctxback_cs_defer_reduction_vs_full_hw"] = _reduction(res, "ctxback_cs_defer")
     res["workload"] = "C1 24-instruction IR kernel, 1 TB x 128 threads, all warps preempted at each of the 24 sites"
+    return res
+
+
+def bench_c2s(cb, trials, seed):
+    """NEXT N2: C2 with shared-memory tiles and barriers; preemption is
+    block-uniform at the barriers and saves each warp's slice of the block's
+    shared memory (8 KiB per TB) with its registers."""
+    import torch
+    from workloads import configs
+    cfg = configs.c2s()
+    progs = _progs(cb, cfg["ir"], min_blocks=2)
+    grid = _grid(progs)
+    dA = torch.from_numpy(cfg["buffers"]["A"].view(np.int32)).cuda()
+    dB = torch.from_numpy(cfg["buffers"]["B"].view(np.int32)).cuda()
+    dC = torch.zeros(4096 * 4096, dtype=torch.int32, device="cuda")
+    ctx = torch.empty(progs["ctxback"].context_capacity(grid), dtype=torch.uint8, device="cuda")
+    run = progs["ctxback"].launch(grid, [dA, dB, dC], [], ctx)
+    run.wait()
+    T = run.launch_ms()
+    ref = dC.clone()
+    del run
+
+    def make():
+        dC.zero_()
+        return [dA, dB, dC]
+    fr = np.random.default_rng(seed + 5).uniform(0.05, 0.95, trials)
+    res = _flag_trials(progs, grid, make, [], lambda b_: bool(torch.equal(b_[2], ref)), fr, T / 1e3)
+    res["static"] = _static(progs["ctxback"], 8)
+    res["static"]["smem_bytes_per_tb"] = 4 * 2048
+    res["reduction_vs_full_hw"] = _reduction(res)
+    res["t_uninterrupted_ms"] = round(T, 3)
+    res["grid"] = grid
+    res["workload"] = ("C2s SGEMM IR 4096^3 with shared-memory k-tiles (8 KiB / TB) and 2 barriers per k-tile; "
+                       "block-uniform preemption at the barriers, flag at U[0.05,0.95] x T")
     return res
 
 
@@ -935,6 +969,7 @@ def gpu_arm(args):
     wanted = [] if args.configs == "none" else [c.strip() for c in args.configs.split(",") if c.strip()]
     for cname in wanted:
         fn = {"c1": lambda: bench_c1(cb), "c3": lambda: bench_c3(cb, args.config_trials, args.seed),
+              "c2s": lambda: bench_c2s(cb, args.config_trials, args.seed),
               "c4a": lambda: bench_c4a(cb, args.config_trials, args.seed),
               "c4b": lambda: bench_c4b(cb, args.config_trials, args.seed),
               "c5": lambda: bench_c5(cb, args.c5_seconds, args.seed, rank)}.get(cname)

@@ -57,7 +57,8 @@ SCA_BYTES = 4     # one uniform 32-bit register per warp       (R-8)
 
 def reexec_op_kind(prog: Program, ins) -> bool:
     """R-4: ALU ops and loads from read-only buffers can be re-executed.
-    Loads from rw buffers, atomics, stores and control flow cannot."""
+    Loads from rw buffers or shared memory (written by other warps), atomics,
+    stores, barriers and control flow cannot."""
     if ins.op in ALU_OPS:
         return True
     if ins.op == "ldg":
@@ -87,7 +88,7 @@ def revert_spec(ins, r):
       'rotl'   : r = rotl(r', k)     (rotr r, r, k; k immediate)
     SHL and every f32 op are irreversible (bits lost / rounding).
     """
-    if ins.dst is None or ins.defreg != r:
+    if ins.dst is None or ins.defreg != r or ins.op == "lds":
         return None
     s = ins.srcs
     regs = [o.reg for o in s if o.is_reg]
@@ -173,8 +174,9 @@ def liveness(prog: Program) -> Liveness:
 def region_heads(prog: Program) -> list:
     """h(c) for every site position c (a global instruction index; the site is
     *before* instruction c).  h(c) = max(BB start, region start), where a new
-    idempotent region starts after every atomic, and *at* a store to buffer b
-    if b was loaded earlier in the current region (memory WAR clobber)."""
+    idempotent region starts after every atomic and every barrier, and *at* a
+    store to buffer b (or shared memory) if b was loaded earlier in the
+    current region (memory WAR clobber)."""
     n = len(prog.instrs)
     heads = [0] * n
     for (s, e) in prog.bbs:
@@ -184,13 +186,13 @@ def region_heads(prog: Program) -> list:
             heads[c] = head
             ins = prog.instrs[c]
             # boundaries triggered by instruction c apply to sites > c
-            if ins.op in ("atom.add", "atom.cas"):
+            if ins.op in ("atom.add", "atom.cas", "bar"):
                 head = c + 1
                 loaded = set()
-            elif ins.op == "stg" and ins.buf in loaded:
+            elif ins.op in ("stg", "sts") and ins.buf in loaded:
                 head = c
                 loaded = set()
-            elif ins.op == "ldg":
+            elif ins.op in ("ldg", "lds"):
                 loaded.add(ins.buf)
     return heads
 
@@ -199,7 +201,12 @@ def sites_for_policy(prog: Program, policy: str, every: int = 8) -> list:
     """Poll-site positions (global instruction indices, site before the instr).
     EVERY_INSTR: before every instruction.  EXPLICIT: the IR's `poll` markers.
     EVERY_N: before BB-local index i for i % N == 0 and i > 0, plus before the
-    terminator of every BB that ends in a backward branch."""
+    terminator of every BB that ends in a backward branch.
+    Kernels with barriers (N2): preemption is block-uniform and fused with a
+    barrier, so the sites are the `bar` instructions (EXPLICIT: the polls, all
+    of which precede a `bar`)."""
+    if prog.has_barriers and policy != "EXPLICIT":
+        return [i for i, ins in enumerate(prog.instrs) if ins.op == "bar"]
     if policy == "EVERY_INSTR":
         return list(range(len(prog.instrs)))
     if policy == "EXPLICIT":
@@ -660,6 +667,17 @@ def _analyze(prog, policy, mode, flags, every, sites, keep_candidates):
 
 def full_ir_bytes(prog):
     return VEC_BYTES * prog.nv + SCA_BYTES * prog.ns
+
+
+def smem_slice(prog, warp):
+    """Shared-memory words warp `warp` of a block saves / restores at a
+    (block-uniform) barrier site: slice = ceil(smem / nwarps) words each."""
+    if prog.smem == 0:
+        return 0, 0
+    sl = -(-prog.smem // prog.nwarps)
+    lo = min(prog.smem, warp * sl)
+    hi = min(prog.smem, lo + sl)
+    return lo, hi
 
 
 def plan_text(prog, pl: Plan) -> str:

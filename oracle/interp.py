@@ -32,7 +32,7 @@ from __future__ import annotations
 import numpy as np
 
 from . import fp32
-from .analysis import PRE, Analysis
+from .analysis import PRE, Analysis, smem_slice
 
 M32 = 0xFFFFFFFF
 NEVER = 0xFFFFFFFF
@@ -204,6 +204,9 @@ class Machine:
         self.sp_lane = np.broadcast_to(lane, (self.nW, 32))
         self.sp_ctaid = (self.warp_ids // nw).astype(np.uint32)
         self.sp_warpid = wib
+        self.nblk = len(self.blocks)
+        self.blk_of = (np.arange(self.nW) // nw).astype(np.int64)     # local block of each warp
+        self.smem = np.zeros((self.nblk, max(1, prog.smem)), dtype=np.uint32)   # zero at block start
         self.records = []          # preemption records
         self.status = np.zeros(self.nW, dtype=np.int8)   # 0 run, 1 parked, 2 done
         self.parked = {}           # local warp -> (c, plan, ctx)
@@ -285,11 +288,30 @@ class Machine:
         if op == "exit":
             self.status[g] = 2
             return []
+        if op == "bar":          # reached only when every warp of the block arrived (_run_gangs)
+            return [(g, pc + 1)]
         a = [self._opd(o, g) for o in ins.srcs]
         guard = self._opd(ins.guard, g) if ins.guard is not None else None
         if op == "ldg":
             val = self._load(ins, g, self._opd(ins.idx, g), guard)
             self._write(ins.defreg, g, val)
+        elif op == "lds":
+            idx = self._full(self._opd(ins.idx, g), n)
+            act = np.ones((n, 32), dtype=bool) if guard is None else (self._full(guard, n) != 0)
+            if np.any(idx[act] >= self.prog.smem):
+                raise OracleError("out-of-bounds shared-memory load")
+            out = np.zeros((n, 32), dtype=np.uint32)
+            rows = np.broadcast_to(self.blk_of[g][:, None], (n, 32))
+            out[act] = self.smem[rows[act], idx[act].astype(np.int64)]
+            self._write(ins.defreg, g, out)
+        elif op == "sts":
+            idx = self._full(self._opd(ins.idx, g), n)
+            val = self._full(a[0], n)
+            act = np.ones((n, 32), dtype=bool) if guard is None else (self._full(guard, n) != 0)
+            if np.any(idx[act] >= self.prog.smem):
+                raise OracleError("out-of-bounds shared-memory store")
+            rows = np.broadcast_to(self.blk_of[g][:, None], (n, 32))
+            self.smem[rows[act], idx[act].astype(np.int64)] = val[act]
         elif op == "stg":
             buf = self.mem[ins.buf]
             idx = self._full(self._opd(ins.idx, g), n)
@@ -359,8 +381,12 @@ class Machine:
                 ctx[v] = np.uint32(self.slot[plan.backup_of[v]][w])
         nbytes = sum(128 if v[0][0] == "v" else 4 for v in ctx)
         assert nbytes == plan.payload_bytes
+        lo, hi = smem_slice(self.prog, int(self.warp_ids[w] % self.prog.nwarps))
+        b = self.blk_of[w]
+        ctx["%smem"] = self.smem[b, lo:hi].copy()
         self.records.append(dict(warp=int(self.warp_ids[w]), site=c, kind=plan.kind,
-                                 bytes=plan.payload_bytes, p=plan.p, launch=self.cur_launch))
+                                 bytes=plan.payload_bytes + 4 * (hi - lo), p=plan.p, launch=self.cur_launch))
+        self.smem[b, lo:hi] = self.rng.integers(0, 1 << 32, hi - lo, dtype=np.uint32)
         # poison every register and slot of the warp (nothing but ctx survives)
         self.V[:, w, :] = self.rng.integers(0, 1 << 32, size=self.V[:, w, :].shape, dtype=np.uint32)
         self.S[:, w] = self.rng.integers(0, 1 << 32, size=self.S[:, w].shape, dtype=np.uint32)
@@ -389,6 +415,8 @@ class Machine:
         """Dedicated resume routine: load, re-execute / revert in schedule
         order (value-SSA), write LIVE_IN(c), continue at c (Figs 2c-6c)."""
         c, plan, ctx = self.parked.pop(w)
+        lo, hi = smem_slice(self.prog, int(self.warp_ids[w] % self.prog.nwarps))
+        self.smem[self.blk_of[w], lo:hi] = ctx.pop("%smem")
         saved_src = {v: src for src, v in plan.saved}
         res = {}     # ('X', j) -> value ; ('R', v) -> value
 
@@ -482,14 +510,30 @@ class Machine:
     # --- launches ------------------------------------------------------------------
     def _run_gangs(self, gangs, targets, count, landing):
         """Run gangs to completion/preemption.  `landing`: local warp -> site
-        it resumed at (no poll there)."""
+        it resumed at (no poll there).  A gang reaching `bar` waits until
+        every running warp of its block has arrived; a poll site at a barrier
+        is decided block-uniformly (any warp's decision preempts the block,
+        as __syncthreads_or does)."""
         prog = self.prog
         ni = len(prog.instrs)
+        gangs = [(g, pc, False) for g, pc in gangs]
+        wait = {}
         while gangs:
-            g, pc = gangs.pop(0)
+            g, pc, released = gangs.pop(0)
             while len(g):
                 if pc >= ni:
                     raise OracleError("fell off the end of the kernel")
+                ins = prog.instrs[pc]
+                if ins.op == "bar" and not released:
+                    for w in g:
+                        wait.setdefault(int(self.blk_of[w]), []).append(int(w))
+                    for b in sorted(set(int(x) for x in self.blk_of[g])):
+                        members = np.nonzero((self.blk_of == b) & (self.status == 0))[0]
+                        if len(wait.get(b, [])) == len(members):
+                            ws = np.array(sorted(wait.pop(b)), dtype=np.int64)
+                            gangs.append((ws, pc, True))
+                    break
+                released = False
                 if landing:
                     land = np.array([landing.get(int(w)) == pc for w in g])
                     for w in g:
@@ -501,6 +545,11 @@ class Machine:
                     if len(pw):
                         hit = count[pw] == targets[pw]
                         count[pw] += 1
+                        if ins.op == "bar":
+                            # block-uniform: OR of the warps' decisions per block
+                            bl = self.blk_of[pw]
+                            anyhit = np.array([hit[bl == b].any() for b in bl])
+                            hit = anyhit
                         pend = self.pend[pw]
                         save = (pend == pc + 1)                      # a deferred preemption lands here
                         start = (pend == 0) & hit
@@ -525,8 +574,10 @@ class Machine:
                 if len(outs) == 1:
                     g, pc = outs[0]
                 else:
-                    gangs[0:0] = outs[1:]
+                    gangs[0:0] = [(x, y, False) for x, y in outs[1:]]
                     g, pc = outs[0]
+        if wait:
+            raise OracleError("warps left waiting at a barrier (non-uniform barrier)")
 
     def run(self, schedule=()):
         """Run launch 0 and as many resume launches as needed.

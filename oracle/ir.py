@@ -86,6 +86,11 @@ class Program:
     labels: dict             # label -> bb index
     explicit_sites: list     # global instruction indices with a 'poll' before them
     bb_succ: list = field(default_factory=list)
+    smem: int = 0            # u32 words of shared memory per block (N2)
+
+    @property
+    def has_barriers(self):
+        return any(i.op == "bar" for i in self.instrs)
 
     @property
     def nwarps(self):
@@ -144,6 +149,7 @@ def parse(text: str) -> Program:
     uniforms: list = []
     nv = ns = None
     block = None
+    smem = 0
     body = []  # (lineno, str)
     for ln, raw in enumerate(text.splitlines(), 1):
         s = raw.split("#", 1)[0].strip()
@@ -162,6 +168,10 @@ def parse(text: str) -> Program:
                 if parts[1] in VECTOR_SPECIALS or parts[1] in UNIFORM_SPECIALS or parts[1] in uniforms:
                     raise IRError(f"line {ln}: bad uniform name {parts[1]}")
                 uniforms.append(parts[1])
+            elif d == ".smem" and len(parts) == 2 and parts[1].isdigit():
+                smem = int(parts[1])
+                if smem > 12288:
+                    raise IRError(f"line {ln}: .smem too large (max 12288 words)")
             elif d in (".vregs", ".sregs", ".block") and len(parts) == 2 and parts[1].isdigit():
                 v = int(parts[1])
                 if d == ".vregs":
@@ -221,6 +231,7 @@ def parse(text: str) -> Program:
         raise IRError("the last instruction must be 'bra' or 'exit'")
 
     prog = Program(name, buffers, uniforms, nv, ns, block, instrs, bbs, labels, explicit_sites)
+    prog.smem = smem
     # validate registers / typing, successors
     succ = []
     for b, (s0, e0) in enumerate(bbs):
@@ -238,6 +249,14 @@ def parse(text: str) -> Program:
     prog.bb_succ = succ
     for ins in instrs:
         _validate(prog, ins)
+    if any(i.op in ("lds", "sts") for i in instrs) and not prog.has_barriers:
+        raise IRError("kernels using shared memory must synchronise with 'bar' "
+                      "(their preemption is block-uniform at barriers)")
+    if prog.has_barriers:
+        for c in explicit_sites:
+            if instrs[c].op != "bar":
+                raise IRError(f"line {instrs[c].line}: in a kernel with barriers, 'poll' may only precede 'bar' "
+                              "(preemption is block-uniform at barriers)")
     return prog
 
 
@@ -331,9 +350,21 @@ def _parse_instr(s, ln, buffers, uniforms):
         if ops:
             raise IRError(f"line {ln}: exit takes no operands")
         ins = Instr("exit")
+    elif opc == "bar":
+        if ops:
+            raise IRError(f"line {ln}: bar takes no operands")
+        ins = Instr("bar")
+    elif opc == "lds":
+        if len(ops) != 2:
+            raise IRError(f"line {ln}: lds d, idx")
+        ins = Instr("lds", dstreg(ops[0]), [], buf="%smem", idx=P(ops[1]))
+    elif opc == "sts":
+        if len(ops) != 2:
+            raise IRError(f"line {ln}: sts idx, a")
+        ins = Instr("sts", None, [P(ops[1])], buf="%smem", idx=P(ops[0]))
     else:
         raise IRError(f"line {ln}: unknown opcode {opc!r}")
-    if guard is not None and ins.op not in ("ldg", "stg", "atom.add", "atom.cas"):
+    if guard is not None and ins.op not in ("ldg", "stg", "atom.add", "atom.cas", "lds", "sts"):
         raise IRError(f"line {ln}: guards only on memory ops")
     ins.guard = guard
     ins.line = ln
@@ -356,6 +387,10 @@ def _validate(prog, ins):
     if ins.op in ("brnz", "brz"):
         if ins.srcs[0].kind != "s":
             raise IRError(f"line {ln}: branch condition must be a scalar register")
+    if ins.op in ("lds", "sts") and prog.smem == 0:
+        raise IRError(f"line {ln}: {ins.op} needs a .smem declaration")
+    if ins.op in ("lds", "sts"):
+        return
     if ins.op == "ldg" and prog.buffers[ins.buf] == "wo":
         raise IRError(f"line {ln}: load from write-only buffer {ins.buf}")
     if ins.op in ("stg", "atom.add", "atom.cas") and prog.buffers[ins.buf] == "ro":

@@ -35,7 +35,8 @@ bool is_alu(Op o) {
   }
 }
 
-// R-4: ALU ops and loads from read-only buffers can be re-executed.
+// R-4: ALU ops and loads from read-only buffers can be re-executed (not loads
+// from rw buffers or shared memory, which other warps write).
 bool reexec_op(const Program& P, const Instr& I) {
   if (is_alu(I.op)) return true;
   if (I.op == Op::Ldg) return P.buf_kinds[I.buf] == B_RO;
@@ -144,14 +145,17 @@ std::vector<int> region_heads(const Program& P) {
     for (int c = s; c < e; c++) {
       heads[c] = head;
       const Instr& I = P.ins[c];
-      if (I.op == Op::AtomAdd || I.op == Op::AtomCas) {
+      const int SMEM_BUF = -2;   // shared memory as one more buffer for the WAR rule
+      if (I.op == Op::AtomAdd || I.op == Op::AtomCas || I.op == Op::Bar) {
         head = c + 1;
         loaded.clear();
-      } else if (I.op == Op::Stg && loaded.count(I.buf)) {
+      } else if ((I.op == Op::Stg && loaded.count(I.buf)) || (I.op == Op::Sts && loaded.count(SMEM_BUF))) {
         head = c;
         loaded.clear();
       } else if (I.op == Op::Ldg) {
         loaded.insert(I.buf);
+      } else if (I.op == Op::Lds) {
+        loaded.insert(SMEM_BUF);
       }
     }
   }
@@ -160,6 +164,11 @@ std::vector<int> region_heads(const Program& P) {
 
 std::vector<int> sites_for(const Program& P, const Options& opt) {
   std::vector<int> out;
+  if (P.has_barriers && opt.policy != 2) {   // block-uniform preemption, fused with the barriers (N2)
+    for (int i = 0; i < (int)P.ins.size(); i++)
+      if (P.ins[i].op == Op::Bar) out.push_back(i);
+    return out;
+  }
   if (opt.policy == 0) {
     for (int i = 0; i < (int)P.ins.size(); i++) out.push_back(i);
   } else if (opt.policy == 2) {

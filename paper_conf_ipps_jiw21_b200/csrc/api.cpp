@@ -73,10 +73,19 @@ struct ctxb_program {
     return num_regs > w ? num_regs - w : 0;
   }
   uint32_t full_hw_bytes() const { return (full_ir_words128() + pad_regs()) * 128u; }
-  uint32_t stride() const {
+  uint32_t smem_slice_bytes() const {
+    if (!prog.smem) return 0;
+    uint32_t nw = (uint32_t)prog.block / 32;
+    return 4u * (((uint32_t)prog.smem + nw - 1) / nw);
+  }
+  uint32_t smem_off() const {   // the warp's smem slice follows its register payload
     uint32_t s = cg.stride;
     if (opt.mode == CTXB_MODE_FULL_HW) s = std::max(s, full_hw_bytes());
-    return std::max<uint32_t>(128, ((s + 127) / 128) * 128);
+    return ((s + 127) / 128) * 128;
+  }
+  uint32_t stride() const {
+    uint32_t s = smem_off() + ((smem_slice_bytes() + 127) / 128) * 128;
+    return std::max<uint32_t>(128, s);
   }
 };
 
@@ -214,7 +223,7 @@ int compile(ctxb_program* p) {
 void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>& blob) {
   size_t nb = std::max<size_t>(1, p->prog.buf_names.size());
   size_t nu = std::max<size_t>(1, p->prog.uniforms.size());
-  size_t words = nb + 5 + (nu + 5 + 1) / 2;
+  size_t words = nb + 5 + (nu + 6 + 1) / 2;
   blob.assign(words, 0);
   for (size_t i = 0; i < r->bufs.size(); i++) blob[i] = r->bufs[i];
   blob[nb + 0] = r->cbuf;
@@ -229,6 +238,7 @@ void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>
   u[nu + 2] = p->pad_regs();
   u[nu + 3] = p->full_hw_bytes();
   u[nu + 4] = 0;   // `zero`: opaque 0 for the timing dependency (gtimer_after)
+  u[nu + 5] = p->smem_off();
 }
 
 int upload_forced(ctxb_run* r, const uint32_t* targets) {

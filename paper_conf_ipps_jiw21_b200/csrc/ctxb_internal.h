@@ -36,6 +36,7 @@ enum class Op : uint8_t {
   FAdd, FSub, FMul,
   FFma, IMad, Sel, Setp,
   Ldg, Stg, AtomAdd, AtomCas,
+  Lds, Sts, Bar,              // shared memory (per block) and the block barrier (N2)
   Bra, Brnz, Brz, Exit
 };
 
@@ -73,6 +74,8 @@ struct Program {
   std::vector<std::vector<int>> succ;     // per BB
   std::map<std::string, int> labels;      // label -> BB
   std::vector<int> explicit_sites;
+  int smem = 0;                           // u32 words of shared memory per block
+  bool has_barriers = false;
   int nregs() const { return nv + ns; }
   bool is_vec(int r) const { return r < nv; }
   std::string regname(int r) const {

@@ -225,10 +225,24 @@ struct Parser {
     } else if (opc == "exit") {
       if (!ops.empty()) fail(line, "exit takes no operands");
       I.op = Op::Exit;
+    } else if (opc == "bar") {
+      if (!ops.empty()) fail(line, "bar takes no operands");
+      I.op = Op::Bar;
+    } else if (opc == "lds") {
+      if (ops.size() != 2) fail(line, "lds d, idx");
+      I.op = Op::Lds;
+      I.dst = dstreg(ops[0]);
+      I.idx = opd(ops[1]);
+    } else if (opc == "sts") {
+      if (ops.size() != 2) fail(line, "sts idx, a");
+      I.op = Op::Sts;
+      I.idx = opd(ops[0]);
+      I.srcs = {opd(ops[1])};
     } else {
       fail(line, "unknown opcode '" + opc + "'");
     }
-    if (guard.kind != OK::None && !(I.op == Op::Ldg || I.op == Op::Stg || I.op == Op::AtomAdd || I.op == Op::AtomCas))
+    if (guard.kind != OK::None && !(I.op == Op::Ldg || I.op == Op::Stg || I.op == Op::AtomAdd || I.op == Op::AtomCas ||
+                                    I.op == Op::Lds || I.op == Op::Sts))
       fail(line, "guards only on memory ops");
     I.guard = guard;
     return I;
@@ -269,6 +283,9 @@ struct Parser {
         } else if (d == ".uniform" && parts.size() == 2) {
           if (reserved(parts[1]) || !is_ident(parts[1])) fail(ln, "bad uniform name " + parts[1]);
           P.uniforms.push_back(parts[1]);
+        } else if (d == ".smem" && parts.size() == 2 && all_digits(parts[1])) {
+          if (parts[1].size() > 6 || std::stoi(parts[1]) > 12288) fail(ln, ".smem too large (max 12288 words)");
+          P.smem = std::stoi(parts[1]);
         } else if ((d == ".vregs" || d == ".sregs" || d == ".block") && parts.size() == 2 && all_digits(parts[1])) {
           if (parts[1].size() > 6) fail(ln, "value too large");
           int v = std::stoi(parts[1]);
@@ -355,6 +372,17 @@ struct Parser {
       P.succ[b].assign(out.begin(), out.end());
     }
     for (auto& I : P.ins) validate(I);
+    bool uses_smem = false;
+    for (auto& I : P.ins) {
+      P.has_barriers = P.has_barriers || I.op == Op::Bar;
+      uses_smem = uses_smem || I.op == Op::Lds || I.op == Op::Sts;
+    }
+    if (uses_smem && !P.has_barriers)
+      throw ParseError("kernels using shared memory must synchronise with 'bar' (their preemption is block-uniform at barriers)");
+    if (P.has_barriers)
+      for (int c : P.explicit_sites)
+        if (P.ins[c].op != Op::Bar)
+          fail(P.ins[c].line, "in a kernel with barriers, 'poll' may only precede 'bar' (preemption is block-uniform at barriers)");
   }
 
   int regid(const Operand& o) const { return o.kind == OK::V ? (int)o.val : P.nv + (int)o.val; }
@@ -378,6 +406,16 @@ struct Parser {
     }
     if ((I.op == Op::Brnz || I.op == Op::Brz) && I.srcs[0].kind != OK::S)
       fail(line, "branch condition must be a scalar register");
+    if ((I.op == Op::Lds || I.op == Op::Sts) && P.smem == 0) fail(line, std::string(I.op == Op::Lds ? "lds" : "sts") + " needs a .smem declaration");
+    if (I.op == Op::Lds || I.op == Op::Sts || I.op == Op::Bar) {
+      I.defreg = I.dst.is_reg() ? regid(I.dst) : -1;
+      I.uses.clear();
+      for (auto& o : I.srcs)
+        if (o.is_reg()) I.uses.push_back(regid(o));
+      if (I.idx.is_reg()) I.uses.push_back(regid(I.idx));
+      if (I.guard.is_reg()) I.uses.push_back(regid(I.guard));
+      return;
+    }
     if (I.op == Op::Ldg && P.buf_kinds[I.buf] == B_WO) fail(line, "load from write-only buffer " + P.buf_names[I.buf]);
     if ((I.op == Op::Stg || I.op == Op::AtomAdd || I.op == Op::AtomCas) && P.buf_kinds[I.buf] == B_RO)
       fail(line, "write to read-only buffer " + P.buf_names[I.buf]);

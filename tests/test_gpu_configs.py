@@ -137,3 +137,76 @@ def test_bulk_save_restore_roundtrip():
     run.resume(forced=np.full(nw, cb.NEVER, np.uint32))
     assert run.wait()
     assert int(out.abs().sum()) == 0
+
+
+def test_c2s_smem_small_forced_block_uniform():
+    """NEXT N2: shared memory + barriers.  Preemption is block-uniform at the
+    barriers (any warp's decision preempts the block); each warp saves its
+    register plan and a slice of the block's shared memory; both are
+    poisoned and restored.  GPU == oracle, headers == oracle records."""
+    cb = _cb()
+    cfg = configs.c2s(128, 128, 32)
+    op = ir.parse(cfg["ir"])
+    an = A.analyze(op, policy="EXPLICIT")
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_FORCED | cb.DEBUG_POISON,
+                      min_blocks_per_sm=2)
+    for k, c in enumerate(an.sites):
+        assert prog.plan_text(k) == A.plan_text(op, an.plans[c])
+    names = list(op.buffers)
+    ref, _ = interp.run(an, 1, cfg["buffers"])
+    g0, _h, _ = gpu_run(prog, names, 1, cfg["buffers"], {})
+    assert np.array_equal(g0["C"], ref["C"])
+    r = np.random.default_rng(8)
+    for _ in range(4):
+        sched = [r.integers(0, 8, 8).astype(np.uint32), r.integers(0, 4, 8).astype(np.uint32)]
+        out, rec = interp.run(an, 1, cfg["buffers"], schedule=sched)
+        assert np.array_equal(out["C"], ref["C"])
+        g, hdrs, _ = gpu_run(prog, names, 1, cfg["buffers"], {}, schedule=sched)
+        assert np.array_equal(g["C"], ref["C"])
+        orc = oracle_records(rec, an)
+        assert header_records(hdrs)[:len(orc)] == orc
+        for launch in orc:                      # block-uniform: all 8 warps of the block together
+            assert len(launch) in (0, 8)
+
+
+def test_c2s_full_flag_equals_c2():
+    import time
+    import torch
+    cb = _cb()
+    cfg = configs.c2s()
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=2)
+    c2p = cb.Program(configs.c2()["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=2)
+    bps, nsm = prog.occupancy()
+    grid = min(bps, c2p.occupancy()[0]) * nsm
+    dA, dB = to_dev(cfg["buffers"]["A"]), to_dev(cfg["buffers"]["B"])
+    dC = torch.zeros(4096 * 4096, dtype=torch.int32, device="cuda")
+    s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
+    ctx2 = torch.zeros(c2p.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    r2 = c2p.launch(grid, [dA, dB, dC], [], ctx2, s)
+    assert r2.wait()
+    ref = dC.clone()
+    ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    dC.zero_()
+    run = prog.launch(grid, [dA, dB, dC], [], ctx, s)
+    assert run.wait()
+    T = run.launch_ms() / 1e3
+    assert torch.equal(dC, ref), "C2s (shared-memory tiles) must equal C2 bit for bit"
+    npre = 0
+    for fr in (0.2, 0.5, 0.8):
+        dC.zero_()
+        torch.cuda.synchronize()
+        run = prog.launch(grid, [dA, dB, dC], [], ctx, s)
+        t0 = time.perf_counter()
+        while time.perf_counter() < t0 + fr * T:
+            pass
+        st = run.preempt(ctrl)
+        npre += st["warps_preempted"]
+        if st["warps_preempted"]:
+            h = run.headers()
+            pre = (h[:, 2] == 1) & (h[:, 3] == 1)
+            assert pre.reshape(-1, 8).all(axis=1).sum() == st["blocks_preempted"]   # whole blocks
+            run.resume(s)
+            assert run.wait()
+        torch.cuda.synchronize()
+        assert torch.equal(dC, ref)
+    assert npre > 0

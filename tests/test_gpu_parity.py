@@ -157,3 +157,16 @@ def test_c2_half_prune_small():
     r = np.random.default_rng(2)
     scheds = [[r.integers(0, 64, 8).astype(np.uint32), r.integers(0, 8, 8).astype(np.uint32)] for _ in range(3)]
     check(cfg["ir"], 1, cfg["buffers"], scheds, policy="EXPLICIT", flags=23)
+
+
+def test_smem_barrier_kernel_block_uniform():
+    """NEXT N2 on the GPU: shared memory + barriers, block-uniform preemption
+    at the barriers (forced per-warp targets OR-ed per block), nested."""
+    import sys, os
+    sys.path.insert(0, os.path.dirname(__file__))
+    from test_smem_oracle import SMEM_K
+    r = np.random.default_rng(1)
+    bufs = {"a": r.integers(0, 1 << 32, 64, dtype=np.uint64).astype(np.uint32), "o": np.zeros(256, np.uint32)}
+    scheds = [[[k] * 6] for k in range(3)] + [[r.integers(0, 3, 6).astype(np.uint32),
+                                               r.integers(0, 2, 6).astype(np.uint32)] for _ in range(6)]
+    check(SMEM_K, 3, bufs, scheds)

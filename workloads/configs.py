@@ -443,3 +443,106 @@ def c5_arrivals(seconds, mean_ms=10.0, seed=51):
     gaps = r.exponential(mean_ms / 1e3, int(seconds / (mean_ms / 1e3) * 3) + 16)
     t = np.cumsum(gaps)
     return t[t < seconds]
+
+
+def c2s_ir(M=4096, N=4096, K=4096):
+    """NEXT N2: C2 with shared-memory tiles and barriers.  Per k-tile of 8 the
+    block stages A (128x8, stored k-major) and B (8x128) in shared memory
+    (4 + 4 loads per thread), `bar`, every thread reads its 8 A and 8 B values
+    per k from shared memory and does 64 FFMAs, `bar`.  Same k order and fma
+    chain as C2, so C is bit-identical to C2's.  Preemption is block-uniform
+    at the two barriers of each k-tile (their windows reach back to the
+    previous barrier)."""
+    assert M % 128 == 0 and N % 128 == 0 and K % 8 == 0
+    tiles_n = N // 128
+    ntiles = (M // 128) * tiles_n
+    L = [".kernel c2s_sgemm_smem", ".buffer ro A", ".buffer ro B", ".buffer wo C",
+         ".vregs 88", ".sregs 7", ".block 256", ".smem 2048"]
+    a, b = 64, 72
+    vA, vB, vT, vC, vty, vtx, vU, vS = 80, 81, 82, 83, 84, 85, 86, 87
+    e = L.append
+    e("init:")
+    e("  mov s0, %ctaid")
+    e(f"  and v{vtx}, %laneid, 15")
+    e(f"  shr v{vty}, %laneid, 4")
+    e("  shl s1, %warpid, 1")
+    e(f"  iadd v{vty}, v{vty}, s1")                  # ty
+    e("tile:")
+    e(f"  setp.lt.u s2, s0, {ntiles}")
+    e("  brz s2, done")
+    e("setup:")
+    shift = tiles_n.bit_length() - 1
+    e(f"  shr s3, s0, {shift}")
+    e(f"  and s4, s0, {tiles_n - 1}")
+    e("  shl s3, s3, 7")                             # row0
+    e("  shl s4, s4, 7")                             # col0
+    # staging indices: A: row0 + tid%128, k0 + (tid/128)*4 + q ; B: k0 + tid/32, col0 + (tid%32)*4 + q
+    e(f"  and v{vT}, %tid, 127")
+    e(f"  iadd v{vA}, v{vT}, s3")
+    e(f"  imul v{vA}, v{vA}, {K}")                   # A row base
+    e(f"  shr v{vU}, %tid, 7")
+    e(f"  shl v{vU}, v{vU}, 2")                      # (tid/128)*4
+    e(f"  iadd v{vA}, v{vA}, v{vU}")                 # A index of (row, k0 + kq)
+    e(f"  shl v{vS}, v{vU}, 7")                      # As offset: kq*128
+    e(f"  iadd v{vS}, v{vS}, v{vT}")                 # As[kq][m]
+    e(f"  shr v{vU}, %tid, 5")                       # kk = tid/32
+    e(f"  imul v{vB}, v{vU}, {N}")
+    e(f"  and v{vT}, %tid, 31")
+    e(f"  shl v{vT}, v{vT}, 2")
+    e(f"  iadd v{vB}, v{vB}, v{vT}")
+    e(f"  iadd v{vB}, v{vB}, s4")                    # B index of (k0 + kk, col0 + 4*(tid%32))
+    e(f"  shl v{vU}, v{vU}, 7")
+    e(f"  iadd v{vU}, v{vU}, v{vT}")
+    e(f"  iadd v{vU}, v{vU}, 1024")                  # Bs[kk][n] at 1024 + kk*128 + n
+    e(f"  iadd v{vC}, v{vty}, s3")
+    e(f"  imul v{vC}, v{vC}, {N}")
+    e(f"  iadd v{vC}, v{vC}, v{vtx}")
+    e(f"  iadd v{vC}, v{vC}, s4")                    # C index of (row0 + ty, col0 + tx)
+    for q in range(64):
+        e(f"  mov v{q}, 0")
+    e(f"  mov s5, {K // 8}")
+    e("ktile:")
+    for q in range(4):                                # stage A: As[kq+q][m]
+        e(f"  iadd v{vT}, v{vA}, {q}")
+        e(f"  ldg v{a + q}, A[v{vT}]")
+        e(f"  iadd v{vT}, v{vS}, {q * 128}")
+        e(f"  sts v{vT}, v{a + q}")
+    for q in range(4):                                # stage B: Bs[kk][n + q]
+        e(f"  iadd v{vT}, v{vB}, {q}")
+        e(f"  ldg v{b + q}, B[v{vT}]")
+        e(f"  iadd v{vT}, v{vU}, {q}")
+        e(f"  sts v{vT}, v{b + q}")
+    e("  poll")
+    e("  bar")
+    for kk in range(8):
+        for i in range(8):
+            e(f"  iadd v{vT}, v{vty}, {kk * 128 + 16 * i}")
+            e(f"  lds v{a + i}, v{vT}")
+        for j in range(8):
+            e(f"  iadd v{vT}, v{vtx}, {1024 + kk * 128 + 16 * j}")
+            e(f"  lds v{b + j}, v{vT}")
+        for q in range(64):
+            i, j = q // 8, q % 8
+            e(f"  ffma v{q}, v{a + i}, v{b + j}, v{q}")
+    e(f"  iadd v{vA}, v{vA}, 8")
+    e(f"  iadd v{vB}, v{vB}, {8 * N}")
+    e("  isub s5, s5, 1")
+    e("  poll")
+    e("  bar")
+    e("  brnz s5, ktile")
+    e("store:")
+    for q in range(64):
+        i, j = q // 8, q % 8
+        e(f"  iadd v{vT}, v{vC}, {16 * i * N + 16 * j}")
+        e(f"  stg C[v{vT}], v{q}")
+    e("  iadd s0, s0, %nctaid")
+    e("  bra tile")
+    e("done:")
+    e("  exit")
+    return "\n".join(L) + "\n"
+
+
+def c2s(M=4096, N=4096, K=4096):
+    cfg = c2(M, N, K)
+    cfg.update(name="C2s", ir=c2s_ir(M, N, K), min_blocks=2)
+    return cfg
