@@ -163,9 +163,12 @@ def parse(text: str) -> Program:
             elif d == ".buffer" and len(parts) == 3 and parts[1] in ("ro", "rw", "wo"):
                 if parts[2] in buffers:
                     raise IRError(f"line {ln}: duplicate buffer {parts[2]}")
+                if not re.fullmatch(r"[A-Za-z_]\w*", parts[2]):
+                    raise IRError(f"line {ln}: bad buffer name")
                 buffers[parts[2]] = parts[1]
             elif d == ".uniform" and len(parts) == 2:
-                if parts[1] in VECTOR_SPECIALS or parts[1] in UNIFORM_SPECIALS or parts[1] in uniforms:
+                if parts[1] in VECTOR_SPECIALS or parts[1] in UNIFORM_SPECIALS or parts[1] in uniforms or \
+                        not re.fullmatch(r"[A-Za-z_]\w*", parts[1]):
                     raise IRError(f"line {ln}: bad uniform name {parts[1]}")
                 uniforms.append(parts[1])
             elif d == ".smem" and len(parts) == 2 and parts[1].isdigit():
@@ -173,6 +176,8 @@ def parse(text: str) -> Program:
                 if smem > 12288:
                     raise IRError(f"line {ln}: .smem too large (max 12288 words)")
             elif d in (".vregs", ".sregs", ".block") and len(parts) == 2 and parts[1].isdigit():
+                if len(parts[1]) > 6:
+                    raise IRError(f"line {ln}: value too large")
                 v = int(parts[1])
                 if d == ".vregs":
                     nv = v
@@ -188,6 +193,8 @@ def parse(text: str) -> Program:
         raise IRError("missing .kernel/.vregs/.sregs/.block")
     if block <= 0 or block % 32 or block > 1024:
         raise IRError(".block must be a positive multiple of 32, <= 1024")
+    if nv > 4096 or ns > 4096:
+        raise IRError("too many registers")
 
     instrs = []
     label_at = {}      # label -> global instr index where it starts
@@ -280,7 +287,10 @@ def _split_ops(rest):
 def _parse_instr(s, ln, buffers, uniforms):
     guard = None
     if s.startswith("@"):
-        g, s = s.split(None, 1)
+        parts = s.split(None, 1)
+        if len(parts) != 2:
+            raise IRError(f"line {ln}: bad guard")
+        g, s = parts
         guard = _parse_opd(g[1:], uniforms, ln)
         if not guard.is_reg:
             raise IRError(f"line {ln}: guard must be a register")
