@@ -421,15 +421,21 @@ def _flag_trials(progs, grid, make_bufs, uniforms, check, fracs, T_s):
             spin_until(time.perf_counter() + fr * T_s)
             st = run.preempt(ctrl)
             rs = {"resume_us": 0.0}
+            save_w = restore_w = None
             if st["warps_preempted"]:
+                hdr = run.headers().copy()
+                pre = (hdr[:, 2] == 1) & (hdr[:, 3] == 1)
                 run.resume(s)
                 run.wait()
                 rs = run.resume_stats()
+                stp = run.stamps()[pre].astype(np.int64)
+                save_w = float(np.median(stp[:, 1] - stp[:, 0])) / 1e3
+                restore_w = float(np.median(stp[:, 3] - stp[:, 2])) / 1e3
             torch.cuda.synchronize()
             if not check(bufs):
                 raise SystemExit(f"{name}: output differs after preempt/resume")
             recs.append(dict(latency_us=st["latency_us"], host_us=st["host_us"], signal_us=st["signal_to_drained_us"],
-                             resume_us=rs["resume_us"],
+                             resume_us=rs["resume_us"], save_warp_us=save_w, restore_warp_us=restore_w,
                              payload=st["payload_bytes"], header=st["header_bytes"], blocks=st["blocks_preempted"],
                              warps=st["warps_preempted"], done=st["warps_done"], step_ms=0.0, launches=2))
             del run
@@ -444,8 +450,8 @@ def _reduction(res, name="ctxback"):
         if c.get(k) and f.get(k):
             return round(100 * (1 - c[k] / f[k]), 2)
         return None
-    return {"latency_pct": pct("latency_us_median"), "resume_pct": pct("resume_us_median"),
-            "context_pct": pct("context_bytes_per_tb")}
+    return {"latency_pct": pct("latency_us_median"), "signal_to_drained_pct": pct("signal_to_drained_us_median"),
+            "resume_pct": pct("resume_us_median"), "context_pct": pct("context_bytes_per_tb")}
 
 
 def bench_c1(cb):
@@ -1001,7 +1007,7 @@ def gpu_arm(args):
     assert torch.equal(hC, ref.cpu()), "e2e result differs"
     e2e_val = float(np.median([x["host_us"] for x in e2e if x["pre"]] or [0.0]))
     # ---- max over ranks ----
-    value = allmax(ws, main["latency_us_median"])
+    value = allmax(ws, main.get("signal_to_drained_us_median") or main["latency_us_median"])
     ms_per_step = allmax(ws, float(np.mean([r["step_ms"] for r in recs])))
     c5_total = None
     if "c5" in extra_cfg:
@@ -1035,13 +1041,22 @@ def gpu_arm(args):
                    "grid": grid, "block": 256, "t_uninterrupted_ms": round(t_unint_ms, 3),
                    "l2": "inputs larger than L2 (A, B, C = 192 MiB > 126 MB)", "parallelism": f"replicas x{ws}"},
         "resume_us": round(main["resume_us_median"], 3),
+        "value_definition": ("median over steps of signal -> all blocks drained: CUDA event on the control stream "
+                             "right before the flag write -> libctxb's event after the victim kernel (every warp "
+                             "saved or finished, kernel exited)"),
+        "preemption_routines_us": round(main["latency_us_median"], 3),
+        "preemption_routines_definition": "max t_saved - min t_flag_seen over preempted warps (%globaltimer)",
         "flag_propagation_us": {"median": round(prop_med, 3), "max": round(prop_max, 3),
                                 "what": "device clock: stamp kernel on the control stream -> cuStreamWriteValue32 "
                                         "-> a spinning warp sees the flag (idle GPU, 20 trials)"},
-        "latency_incl_flag_propagation_us": round(value + prop_med, 3),
+        "routines_plus_flag_propagation_us": round(main["latency_us_median"] + prop_med, 3),
         "context_bytes_per_tb": main.get("context_bytes_per_tb"),
         "ctxback": main, "baselines": base, "static_context": static,
         "reduction_vs_full_hw": {
+            "signal_to_drained_pct": (round(100 * (1 - main["signal_to_drained_us_median"] /
+                                                   base["full_hw"]["signal_to_drained_us_median"]), 2)
+                                      if "full_hw" in base and base["full_hw"].get("signal_to_drained_us_median")
+                                      else None),
             "latency_pct": (round(100 * (1 - main["latency_us_median"] / base["full_hw"]["latency_us_median"]), 2)
                             if "full_hw" in base and base["full_hw"]["latency_us_median"] else None),
             "resume_pct": (round(100 * (1 - main["resume_us_median"] / base["full_hw"]["resume_us_median"]), 2)

@@ -92,6 +92,10 @@ extern "C" {
 #define CTXB_DEBUG_NO_COMPILE 8u /* analysis + code generation only            */
 #define CTXB_DEBUG_NO_SHARE  16u /* one preemption routine per site (no P:317
                                     sharing of identical routines)             */
+#define CTXB_DEBUG_FENCE_STAMPS 32u /* __threadfence before the t_saved stamp, so
+                                    it marks the payload as visible (slower
+                                    drain; by default the kernel boundary orders
+                                    the context for the resume launch)          */
 
 typedef struct {
   uint32_t flags;       /* CTXB_RELAXED | CTXB_REVERT | CTXB_OSRB                */
@@ -147,8 +151,9 @@ typedef struct {
 
 typedef struct {
   double latency_us;         /* device: max t_saved - min t_flag_seen over preempted
-                                warps (%globaltimer), "elapsed time before
-                                releasing the GPU"                                 */
+                                warps (%globaltimer): the preemption routines'
+                                span (t_saved = stores issued; with
+                                CTXB_DEBUG_FENCE_STAMPS: stores visible)          */
   double host_us;            /* host: flag write issued -> victim stream drained   */
   double signal_to_drained_us; /* CUDA events: event on ctrl right before the flag
                                 write -> the library's event after the victim

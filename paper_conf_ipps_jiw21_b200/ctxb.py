@@ -16,7 +16,7 @@ __all__ = [
     "LIB_PATH", "CtxbError", "lib",
     "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
-    "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE",
+    "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "EXPORTED_SYMBOLS",
     "ctxb_analyze", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait", "ctxb_context_bytes",
     "ctxb_flag_propagation",
@@ -29,6 +29,7 @@ RELAXED, REVERT, OSRB, ALL, DEFER, PRUNE = 1, 2, 4, 7, 8, 16
 MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
 DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1, 2, 4, 8, 16
+DEBUG_FENCE_STAMPS = 32
 STATE_NONE, STATE_PREEMPTED, STATE_DONE = 0, 1, 2
 NEVER = 0xFFFFFFFF
 
