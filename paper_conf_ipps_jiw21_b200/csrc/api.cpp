@@ -615,7 +615,7 @@ static __device__ __forceinline__ u64 gt() { u64 t; asm volatile("mov.u64 %0, %%
 static __device__ __forceinline__ u32 ldcv(const u32* p) { u32 v; asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p)); return v; }
 extern "C" __global__ void ctxb_probe_spin(const u32* flag, u64* out) {
   u64 t0 = gt();
-  while (ldcv(flag) == 0u) { if (gt() - t0 > 2000000000ull) break; }
+  while (ldcv(flag) == 0u) { if (gt() - t0 > 20000000ull) break; }   // 20 ms timeout
   if (threadIdx.x == 0) out[1] = gt();
 }
 extern "C" __global__ void ctxb_probe_stamp(u64* out) { if (threadIdx.x == 0) out[0] = gt(); }
