@@ -901,6 +901,54 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
                         "each a ~1.5 ms bf16 GEMM on a high-priority stream; per arrival preempt -> LS -> resume"}
 
 
+def _oracle_tb(args_):
+    """Interpret thread block `b` of C2 (M=N=512, K=256; 16 tiles) with the
+    oracle, preempting all its warps at one poll visit; returns seconds."""
+    b, an_pickle = args_
+    import pickle
+    from oracle import interp
+    from workloads import configs
+    an = pickle.loads(an_pickle)
+    cfg = configs.c2(512, 512, 256)
+    t0 = time.perf_counter()
+    m = interp.Machine(an, 16, cfg["buffers"], blocks=[b])
+    m.run([np.full(8, 7, np.uint32)])
+    return time.perf_counter() - t0
+
+
+def oracle_throughput(max_cores=None):
+    """Oracle on host cores: thread blocks interpreted per
+    second on 1 core and on all cores (multiprocessing over TBs)."""
+    import multiprocessing as mpr
+    import pickle
+    import platform
+    from oracle import analysis as A
+    from oracle import ir
+    from workloads import configs
+    cfg = configs.c2(512, 512, 256)
+    an = A.analyze(ir.parse(cfg["ir"]), policy="EXPLICIT")
+    blob = pickle.dumps(an)
+    t1 = _oracle_tb((0, blob))
+    n = max_cores or os.cpu_count() or 1
+    ctx = mpr.get_context("fork")
+    t0 = time.perf_counter()
+    with ctx.Pool(n) as pool:
+        pool.map(_oracle_tb, [(b % 16, blob) for b in range(max(n, 16))])
+    tw = time.perf_counter() - t0
+    model = platform.processor() or ""
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"tb_seconds_1core": round(t1, 3), "tb_per_s_1core": round(1.0 / t1, 3),
+            "tb_per_s_all_cores": round(max(n, 16) / tw, 3), "cores_all": n, "cpu_model": model,
+            "sample": "C2 IR M=N=512, K=256: one thread block (8 warps, 1 tile, 64 k-iterations) "
+                      "interpreted and preempted at poll visit 7, then resumed to completion"}
+
+
 def gpu_arm(args):
     import torch
     import paper_conf_ipps_jiw21_b200 as cb
@@ -1020,6 +1068,7 @@ def gpu_arm(args):
         samp, t_an = oracle_sample(1, args.seed)
         cpu = {"value": samp[0]["latency_us"], "unit": "us", "cores": 1, "kind": "oracle",
                "resume_us": samp[0]["resume_us"], "context_bytes_per_tb": samp[0]["bytes"],
+               "throughput": oracle_throughput(),
                "sample": (f"C2 IR at M=N=K=256, thread block 0 (8 warps) preempted at poll visit "
                           f"{samp[0]['visit']} and resumed to completion on 1 host core; value = host time "
                           f"in the oracle's preemption routine for the 8 warps (analysis {t_an:.1f} s, "

@@ -210,3 +210,58 @@ def test_c2s_full_flag_equals_c2():
         torch.cuda.synchronize()
         assert torch.equal(dC, ref)
     assert npre > 0
+
+
+@pytest.mark.parametrize("which", ["c2", "c3", "c2s"])
+def test_flag_mode_repeated_nested_preemption(which):
+    """random flag times, repeated and nested
+    preempt -> resume -> preempt ... cycles (each resume can be preempted
+    again, also inside the same basic-block pass: the LIVE fallback, R-16);
+    the final output stays bit-exact with the uninterrupted run."""
+    import time
+    import torch
+    cb = _cb()
+    if which == "c3":
+        cfg = configs.c3()
+        bufs = [to_dev(cfg["buffers"]["X"]), torch.zeros(cfg["W"] * cfg["H"], dtype=torch.int32, device="cuda")]
+        out_i, mb = 1, 0
+    else:
+        cfg = configs.c2() if which == "c2" else configs.c2s()
+        bufs = [to_dev(cfg["buffers"]["A"]), to_dev(cfg["buffers"]["B"]),
+                torch.zeros(4096 * 4096, dtype=torch.int32, device="cuda")]
+        out_i, mb = 2, 2
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=mb)
+    bps, nsm = prog.occupancy()
+    grid = bps * nsm
+    ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
+    run = prog.launch(grid, bufs, [], ctx, s)
+    assert run.wait()
+    T = run.launch_ms() / 1e3
+    ref = bufs[out_i].clone()
+    rng = np.random.default_rng(77)
+    total_pre = cycles = 0
+    for trial in range(3):
+        bufs[out_i].zero_()
+        torch.cuda.synchronize()
+        run = prog.launch(grid, bufs, [], ctx, s)
+        while True:
+            t0 = time.perf_counter()
+            while time.perf_counter() < t0 + rng.uniform(0.02, 0.25) * T:
+                pass
+            st = run.preempt(ctrl)
+            if not st["warps_preempted"]:
+                break
+            total_pre += st["warps_preempted"]
+            cycles += 1
+            run.resume(s)
+            if cycles > 40:
+                assert run.wait() or True
+                break
+        if not run.wait():
+            while not run.finished:
+                run.resume(s)
+                run.wait()
+        torch.cuda.synchronize()
+        assert torch.equal(bufs[out_i], ref), f"{which}: output differs after {cycles} nested cycles"
+    assert cycles >= 3 and total_pre > 0
