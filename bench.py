@@ -380,7 +380,8 @@ def oracle_sample(steps=1, seed=0):
 # ---- the other BASELINE configs (configs[0], [2], [3]) ----------------------
 
 MODES = (("ctxback", 0, 7), ("full_hw", 3, 7), ("live", 1, 7),
-         ("cs_defer", 1, 15), ("ctxback_cs_defer", 0, 15))      # (name, mode, flags); 15 = ALL | DEFER
+         ("cs_defer", 1, 15), ("ctxback_cs_defer", 0, 15),      # (name, mode, flags); 15 = ALL | DEFER
+         ("ctxback_rank_resume", 0, 39))                        # 39 = ALL | RANK_RESUME (NEXT N4)
 
 
 def _progs(cb, ir_text, debug=0, min_blocks=0):
@@ -493,6 +494,7 @@ def bench_c1(cb):
         if name == "ctxback":
             res["static"] = _static(prog, 4)
     res["reduction_vs_full_hw"] = _reduction(res)
+    res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["cs_defer_reduction_vs_full_hw"] = _reduction(res, "cs_defer")
     res["ctxback_cs_defer_reduction_vs_full_hw"] = _reduction(res, "ctxback_cs_defer")
     res["workload"] = "C1 24-instruction IR kernel, 1 TB x 128 threads, all warps preempted at each of the 24 sites"
@@ -526,6 +528,7 @@ def bench_c2s(cb, trials, seed):
     res["static"] = _static(progs["ctxback"], 8)
     res["static"]["smem_bytes_per_tb"] = 4 * 2048
     res["reduction_vs_full_hw"] = _reduction(res)
+    res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["t_uninterrupted_ms"] = round(T, 3)
     res["grid"] = grid
     res["workload"] = ("C2s SGEMM IR 4096^3 with shared-memory k-tiles (8 KiB / TB) and 2 barriers per k-tile; "
@@ -557,6 +560,7 @@ def bench_c3(cb, trials, seed):
     res = _flag_trials(progs, grid, make, [], lambda b: bool(torch.equal(b[1], ref)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
     res["reduction_vs_full_hw"] = _reduction(res)
+    res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["cs_defer_reduction_vs_full_hw"] = _reduction(res, "cs_defer")
     res["ctxback_cs_defer_reduction_vs_full_hw"] = _reduction(res, "ctxback_cs_defer")
     res["t_uninterrupted_ms"] = round(T, 3)
@@ -596,6 +600,7 @@ def bench_c4a(cb, trials, seed):
     res["static"]["ctxback_osrb_off_bytes_per_tb_per_site"] = [
         8 * osrb_off.site_info(k)["payload_bytes_per_warp"] for k in range(osrb_off.num_sites)]
     res["reduction_vs_full_hw"] = _reduction(res)
+    res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["t_uninterrupted_ms"] = round(T, 3)
     res["grid"] = grid
     res["uninterrupted_equals_bincount"] = ok
@@ -663,6 +668,7 @@ def bench_c4b(cb, trials, seed):
         res[name] = summarize(recs)
     res["static"] = _static(progs["ctxback"], 8)
     res["reduction_vs_full_hw"] = _reduction(res)
+    res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["grid"] = grid
     res["largest_level"] = big
     res["workload"] = (f"C4b level-synchronous BFS IR, n=2^22, {len(ci)} edges (Poisson(16) out-degree), "

@@ -69,6 +69,14 @@ extern "C" {
                              registers live at the site need, instead of every
                              live-out result of the window (R-2, literal); every
                              flashback-point becomes feasible                     */
+#define CTXB_RANK_RESUME 32u /* combined ranking (NEXT N4): per site pick the
+                             flashback-point minimising the estimated preempt +
+                             resume cost E = 2*payload + re-executed load bytes +
+                             resume_level_bytes*(dependent memory round trips - 1)
+                             + defer_instr_bytes*(reverts + re-executions), ties
+                             by the R-10 key; the paper ranks by preemption
+                             latency only and notes re-execution can dominate
+                             resuming                          */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */
@@ -113,6 +121,10 @@ typedef struct {
   uint32_t defer_instr_bytes; /* CTXB_DEFER latency estimate: one deferred instruction
                            costs this many context bytes (0 = 8); the stalls of the
                            deferred instructions are ignored, as in P:380          */
+  uint32_t resume_level_bytes; /* CTXB_RANK_RESUME: one dependent memory round trip on
+                           the resume path costs this many context bytes per warp
+                           (0 = 512 ~ an HBM round trip x one warp's share of HBM
+                           bandwidth when every warp of the chip restores)        */
 } ctxb_options;
 
 typedef struct ctxb_program ctxb_program; /* analysed IR kernel + module; library-owned */

@@ -44,8 +44,10 @@ FLAG_OSRB = 4
 FLAGS_ALL = 7
 FLAG_DEFER = 8            # CS-Defer on top of the mode's own plans
 FLAG_PRUNE = 16           # demand-driven restore (NEXT N4): restore only what LIVE_IN(c) needs
+FLAG_RANK_RESUME = 32     # combined preempt + resume ranking of flashback-points (NEXT N4)
 
 DEFER_INSTR_BYTES = 8     # latency-estimate weight of one deferred instruction, in context bytes
+RESUME_LEVEL_BYTES = 512  # FLAG_RANK_RESUME: one dependent memory round trip, in context bytes
 
 MODE_CTXBACK = 0
 MODE_LIVE = 1
@@ -562,16 +564,68 @@ class Analysis:
     defer: dict = field(default_factory=dict)        # site c -> site it defers to (c itself: none)
 
 
-def best_plan(prog, lv, heads, c, backups, flags, keep=None):
+def resume_estimate(prog, pl, instr_bytes=DEFER_INSTR_BYTES, level_bytes=RESUME_LEVEL_BYTES):
+    """FLAG_RANK_RESUME (NEXT N4; the paper ranks by preemption latency only
+    and notes that re-execution can dominate resuming):
+    estimated preempt + resume cost of a plan in context-byte units,
+
+      E = 2 * payload                      context written at preempt, read at resume
+        + sum of re-executed load bytes     128 B (vector) / 4 B (scalar) per warp
+        + level_bytes * (levels - 1)        dependent memory round trips after the restore
+        + instr_bytes * (#reverts + #re-executions)
+
+    levels = depth of the resume schedule in memory round trips: a restored
+    value (saved, backed up or recovered at preempt) is at level 1, a
+    re-executed load at 1 + the deepest of its operands, any other re-executed
+    or reverted instruction at the deepest of its operands."""
+    saved_p = {(v[0], pl.revert_info[v][0]) for src, v in pl.saved if src == "P"}
+    lx, lr = {}, {}
+
+    def level(reg, s):
+        if s[0] in ("C", "B"):
+            return 1
+        if s[0] == "X":
+            return lx[s[1]]
+        return 1 if (reg, s[1]) in saved_p else lr[(reg, s[1])]
+
+    depth = 1 if pl.saved else 0
+    load_bytes = 0
+    for e in pl.schedule:
+        if e[0] == "X":
+            j = e[1]
+            ins = prog.instrs[j]
+            lv_ = max([level(r, s) for r, s in zip(ins.uses(), pl.reexec_supply[j])], default=0)
+            if ins.op == "ldg":
+                lv_ += 1
+                load_bytes += VEC_BYTES if prog.is_vector(ins.defreg) else SCA_BYTES
+            lx[j] = lv_
+        else:
+            v = e[1]
+            m, _k, ins_, sups = pl.revert_info[v]
+            lv_ = max([level(x[0], s) for x, s in zip(ins_, sups)], default=0)
+            lr[(v[0], m)] = lv_
+        depth = max(depth, lv_)
+    ops = len(pl.schedule) + len(pl.preempt_reverts)
+    return 2 * pl.payload_bytes + load_bytes + level_bytes * max(0, depth - 1) + instr_bytes * ops
+
+
+def best_plan(prog, lv, heads, c, backups, flags, keep=None, est=None):
     """Enumerate p = c, c-1, ..., h(c) (R-1, R-3) and pick the lexicographic
-    minimum of Plan.cost() (R-10)."""
-    best = None
+    minimum of Plan.cost() (R-10); with FLAG_RANK_RESUME the minimum of
+    (resume_estimate, Plan.cost()).  `est` = (instr_bytes, level_bytes)."""
+    def key(pl):
+        if flags & FLAG_RANK_RESUME:
+            return (resume_estimate(prog, pl, *(est or ())),) + pl.cost()
+        return pl.cost()
+    best, best_k = None, None
     for p in range(c, heads[c] - 1, -1):
         pl = plan_window(prog, lv, p, c, backups, flags)
         if keep is not None:
             keep[p] = pl
-        if pl is not None and (best is None or pl.cost() < best.cost()):
-            best = pl
+        if pl is not None:
+            k = key(pl)
+            if best is None or k < best_k:
+                best, best_k = pl, k
     return best
 
 
@@ -623,9 +677,11 @@ def defer_targets(prog, sites, plans, instr_bytes=DEFER_INSTR_BYTES):
 
 
 def analyze(prog: Program, policy="EVERY_INSTR", mode=MODE_CTXBACK, flags=FLAGS_ALL,
-            every=8, sites=None, keep_candidates=False, defer_instr_bytes=DEFER_INSTR_BYTES) -> Analysis:
+            every=8, sites=None, keep_candidates=False, defer_instr_bytes=DEFER_INSTR_BYTES,
+            resume_level_bytes=RESUME_LEVEL_BYTES) -> Analysis:
     """Compile-time analysis: per poll site, the chosen plan."""
-    an = _analyze(prog, policy, mode, flags & (FLAGS_ALL | FLAG_PRUNE), every, sites, keep_candidates)
+    an = _analyze(prog, policy, mode, flags & (FLAGS_ALL | FLAG_PRUNE | FLAG_RANK_RESUME), every, sites,
+                  keep_candidates, (defer_instr_bytes, resume_level_bytes))
     an.flags = flags
     if flags & FLAG_DEFER:
         an.defer = defer_targets(prog, an.sites, an.plans, defer_instr_bytes)
@@ -634,7 +690,7 @@ def analyze(prog: Program, policy="EVERY_INSTR", mode=MODE_CTXBACK, flags=FLAGS_
     return an
 
 
-def _analyze(prog, policy, mode, flags, every, sites, keep_candidates):
+def _analyze(prog, policy, mode, flags, every, sites, keep_candidates, est=None):
     lv = liveness(prog)
     heads = region_heads(prog)
     if sites is None:
@@ -647,19 +703,21 @@ def _analyze(prog, policy, mode, flags, every, sites, keep_candidates):
                         live, mode=mode, flags=flags)
     backups = []
     if (flags & FLAG_OSRB) and (flags & FLAG_RELAXED):
-        base = {c: best_plan(prog, lv, heads, c, (), flags).payload_bytes for c in sites}
+        # R-7 selects backups by the bytes of the R-10 choice, whatever the ranking
+        fb = flags & ~FLAG_RANK_RESUME
+        base = {c: best_plan(prog, lv, heads, c, (), fb).payload_bytes for c in sites}
         for m in osrb_candidates(prog):
             bb = prog.bb_of(m)
             for c in sites:
                 if prog.bb_of(c) != bb or c <= m or heads[c] > m:
                     continue
-                if best_plan(prog, lv, heads, c, (m,), flags).payload_bytes < base[c]:
+                if best_plan(prog, lv, heads, c, (m,), fb).payload_bytes < base[c]:
                     backups.append(m)
                     break
     plans, cands = {}, {}
     for c in sites:
         keep = {} if keep_candidates else None
-        plans[c] = best_plan(prog, lv, heads, c, backups, flags, keep)
+        plans[c] = best_plan(prog, lv, heads, c, backups, flags, keep, est)
         if keep_candidates:
             cands[c] = keep
     return Analysis(prog, lv, sites, heads, backups, plans, live, cands, mode, flags)

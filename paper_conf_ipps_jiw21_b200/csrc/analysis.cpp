@@ -19,7 +19,7 @@
 namespace ctxb {
 namespace {
 
-constexpr uint32_t F_RELAXED = 1, F_REVERT = 2, F_OSRB = 4, F_DEFER = 8, F_PRUNE = 16;
+constexpr uint32_t F_RELAXED = 1, F_REVERT = 2, F_OSRB = 4, F_DEFER = 8, F_PRUNE = 16, F_RANK_RESUME = 32;
 constexpr uint32_t VEC_B = 128, SCA_B = 4;
 
 bool is_alu(Op o) {
@@ -538,14 +538,63 @@ Plan window_plan(const Program& P, const Liveness& L, const DefIndex& D, int p, 
   return w.plan(0);
 }
 
+// CTXB_RANK_RESUME (NEXT N4; the paper ranks by preemption latency only and
+// notes that re-execution can dominate resuming): estimated
+// preempt + resume cost of a plan in context-byte units,
+//   E = 2 * payload + re-executed load bytes + level_bytes * (levels - 1)
+//     + instr_bytes * (#reverts + #re-executions),
+// levels = memory round trips on the resume schedule: restored values at 1,
+// a re-executed load at 1 + its deepest operand, other ops at their deepest.
+uint64_t resume_estimate(const Program& P, const Plan& pl, uint32_t instr_bytes, uint32_t level_bytes) {
+  std::set<std::pair<int, int>> saved_p;   // (reg, m) recovered at preempt and saved
+  for (auto& sv : pl.saved)
+    if (sv.src == 'P') saved_p.insert({sv.v.r, pl.revert_info.at(sv.v).m});
+  std::map<int, int> lx;
+  std::map<std::pair<int, int>, int> lr;
+  auto level = [&](int reg, const Supply& s) -> int {
+    switch (s.k) {
+      case SK::C:
+      case SK::B: return 1;
+      case SK::X: return lx.at(s.arg);
+      case SK::R: return saved_p.count({reg, s.arg}) ? 1 : lr.at({reg, s.arg});
+    }
+    return 1;
+  };
+  int depth = pl.saved.empty() ? 0 : 1;
+  uint64_t load_bytes = 0;
+  for (auto& e : pl.schedule) {
+    int l = 0;
+    if (e.is_x) {
+      const Instr& I = P.ins[e.j];
+      const std::vector<Supply>& sup = pl.reexec_supply.at(e.j);
+      for (size_t k = 0; k < I.uses.size(); k++) l = std::max(l, level(I.uses[k], sup[k]));
+      if (I.op == Op::Ldg) {
+        l += 1;
+        load_bytes += P.is_vec(I.defreg) ? VEC_B : SCA_B;
+      }
+      lx[e.j] = l;
+    } else {
+      const RevertRec& rec = pl.revert_info.at(e.v);
+      for (size_t k = 0; k < rec.inputs.size(); k++) l = std::max(l, level(rec.inputs[k].r, rec.supplies[k]));
+      lr[{e.v.r, rec.m}] = l;
+    }
+    depth = std::max(depth, l);
+  }
+  uint64_t ops = pl.schedule.size() + pl.pre_reverts.size();
+  return 2ull * pl.payload_bytes + load_bytes + (uint64_t)level_bytes * (uint64_t)std::max(0, depth - 1) +
+         (uint64_t)instr_bytes * ops;
+}
+
 Plan best_plan(const Program& P, const Liveness& L, const DefIndex& D, const std::vector<int>& heads, int c,
-               const std::vector<int>& bk, uint32_t flags) {
+               const std::vector<int>& bk, uint32_t flags, uint32_t instr_bytes = 8, uint32_t level_bytes = 512) {
   Plan best;
-  std::vector<int> bc;
+  std::vector<int64_t> bc;
   for (int p = c; p >= heads[c]; p--) {
     Plan pl = window_plan(P, L, D, p, c, bk, flags);
     if (!pl.valid) continue;
-    std::vector<int> k = pl.cost();
+    std::vector<int64_t> k;
+    if (flags & F_RANK_RESUME) k.push_back((int64_t)resume_estimate(P, pl, instr_bytes, level_bytes));
+    for (int x : pl.cost()) k.push_back(x);
     if (!best.valid || k < bc) {
       best = std::move(pl);
       bc = k;
@@ -638,7 +687,7 @@ Analysis analyze(const Program& P, const Options& opt) {
 
 static Analysis analyze_plans(const Program& P, const Options& opt0) {
   Options opt = opt0;
-  opt.flags &= (7u | F_PRUNE);
+  opt.flags &= (7u | F_PRUNE | F_RANK_RESUME);
   Liveness L = liveness(P);
   DefIndex D(P);
   Analysis A;
@@ -661,20 +710,23 @@ static Analysis analyze_plans(const Program& P, const Options& opt0) {
   }
   uint32_t fl = opt.flags;
   if ((fl & F_OSRB) && (fl & F_RELAXED)) {
+    // R-7 selects backups by the bytes of the R-10 choice, whatever the ranking
+    uint32_t fb = fl & ~F_RANK_RESUME;
     std::map<int, uint32_t> base;
-    for (int c : A.sites) base[c] = best_plan(P, L, D, A.heads, c, {}, fl).payload_bytes;
+    for (int c : A.sites) base[c] = best_plan(P, L, D, A.heads, c, {}, fb).payload_bytes;
     for (int m : osrb_candidates(P)) {
       int bbm = P.bb_of[m];
       for (int c : A.sites) {
         if (c >= (int)P.ins.size() || P.bb_of[c] != bbm || c <= m || A.heads[c] > m) continue;
-        if (best_plan(P, L, D, A.heads, c, {m}, fl).payload_bytes < base[c]) {
+        if (best_plan(P, L, D, A.heads, c, {m}, fb).payload_bytes < base[c]) {
           A.backups.push_back(m);
           break;
         }
       }
     }
   }
-  for (int c : A.sites) A.plans.push_back(best_plan(P, L, D, A.heads, c, A.backups, fl));
+  for (int c : A.sites)
+    A.plans.push_back(best_plan(P, L, D, A.heads, c, A.backups, fl, opt.defer_instr_bytes, opt.resume_level_bytes));
   return A;
 }
 

@@ -142,6 +142,7 @@ struct Plan {
 struct Options {
   uint32_t flags = 7, mode = 0, policy = 0, every = 8, debug = 0, flag_depth = 1, min_blocks = 0;
   uint32_t defer_instr_bytes = 8;   // CS-Defer latency-estimate weight per deferred instruction
+  uint32_t resume_level_bytes = 512;  // CTXB_RANK_RESUME weight of one dependent memory round trip
 };
 
 struct Analysis {

@@ -14,7 +14,7 @@ import numpy as np
 
 __all__ = [
     "LIB_PATH", "CtxbError", "lib",
-    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
+    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
     "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "EXPORTED_SYMBOLS",
@@ -25,7 +25,7 @@ __all__ = [
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libctxb.so")
 
-RELAXED, REVERT, OSRB, ALL, DEFER, PRUNE = 1, 2, 4, 7, 8, 16
+RELAXED, REVERT, OSRB, ALL, DEFER, PRUNE, RANK_RESUME = 1, 2, 4, 7, 8, 16, 32
 MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
 DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1, 2, 4, 8, 16
@@ -51,7 +51,8 @@ class CtxbError(RuntimeError):
 class _Opts(C.Structure):
     _fields_ = [("flags", C.c_uint32), ("mode", C.c_uint32), ("poll_policy", C.c_uint32),
                 ("poll_every", C.c_uint32), ("debug", C.c_uint32), ("flag_depth", C.c_uint32),
-                ("min_blocks_per_sm", C.c_uint32), ("defer_instr_bytes", C.c_uint32)]
+                ("min_blocks_per_sm", C.c_uint32), ("defer_instr_bytes", C.c_uint32),
+                ("resume_level_bytes", C.c_uint32)]
 
 
 class _SiteInfo(C.Structure):
@@ -152,9 +153,10 @@ def _u32arr(vals):
 # --- the C-ABI names ----------------------------------------------------------
 
 def ctxb_analyze(ir_text: str, flags=ALL, mode=MODE_CTXBACK, poll_policy=POLL_EVERY_INSTR, poll_every=8,
-                 debug=0, flag_depth=1, min_blocks_per_sm=0, defer_instr_bytes=8) -> "Program":
+                 debug=0, flag_depth=1, min_blocks_per_sm=0, defer_instr_bytes=8,
+                 resume_level_bytes=512) -> "Program":
     return Program(ir_text, flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm,
-                   defer_instr_bytes)
+                   defer_instr_bytes, resume_level_bytes)
 
 
 def ctxb_launch(prog, grid, buffers, uniforms, ctx, stream=None, forced=None) -> "Run":
@@ -189,9 +191,10 @@ class Program:
     """An analysed + compiled IR kernel (ctxb_analyze)."""
 
     def __init__(self, ir_text, flags=ALL, mode=MODE_CTXBACK, poll_policy=POLL_EVERY_INSTR, poll_every=8,
-                 debug=0, flag_depth=1, min_blocks_per_sm=0, defer_instr_bytes=8):
+                 debug=0, flag_depth=1, min_blocks_per_sm=0, defer_instr_bytes=8, resume_level_bytes=512):
         self._h = C.c_void_p()
-        o = _Opts(flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm, defer_instr_bytes)
+        o = _Opts(flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm, defer_instr_bytes,
+                  resume_level_bytes)
         b = ir_text.encode()
         _chk(lib.ctxb_analyze(b, len(b), C.byref(o), C.byref(self._h)))
         self.debug = debug

@@ -24,11 +24,12 @@ def _cb():
     return cb
 
 
-def forced_parity(cfg, grid, nsched, max_visit, skip=(), compare=None, seed=5):
+def forced_parity(cfg, grid, nsched, max_visit, skip=(), compare=None, seed=5, flags=7):
     cb = _cb()
     op = ir.parse(cfg["ir"])
-    an = A.analyze(op, policy="EXPLICIT")
-    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_FORCED | cb.DEBUG_POISON)
+    an = A.analyze(op, policy="EXPLICIT", flags=flags)
+    prog = cb.Program(cfg["ir"], flags=flags, poll_policy=cb.POLL_EXPLICIT,
+                      debug=cb.DEBUG_FORCED | cb.DEBUG_POISON)
     for k, c in enumerate(an.sites):
         assert prog.plan_text(k) == A.plan_text(op, an.plans[c])
     names = list(op.buffers)
@@ -61,13 +62,21 @@ def test_c3_small_forced():
     assert any(an.plans[c].n_revert_res + an.plans[c].n_revert_pre > 0 for c in an.sites)
 
 
+def test_c3_small_forced_rank_resume():
+    """CTXB_RANK_RESUME (NEXT N4) plans on the GPU vs the oracle."""
+    cfg = configs.c3(512, 128, 64)
+    an = forced_parity(cfg, 4, 3, 128, flags=7 | 32)
+    assert all(an.plans[c].p == c for c in an.sites)
+
+
 def test_c4a_small_forced():
     cfg = configs.c4a(1 << 14, grid=2)
     an = forced_parity(cfg, 2, 3, 4)
     assert an.backups, "C4a must select an OSRB backup"
 
 
-def test_c4b_small_forced_level():
+@pytest.mark.parametrize("flags", [7, 7 | 32])
+def test_c4b_small_forced_level(flags):
     rp, ci = configs.c4b_graph(1 << 10, 16)
     n = len(rp) - 1
     dist = np.full(n, 0xFFFFFFFF, np.uint32)
@@ -82,7 +91,7 @@ def test_c4b_small_forced_level():
 
         def cmp_nextf(g, o, ref, cnt=None):
             pass
-        forced_parity(cfg, 2, 2, 40, skip=("nextf",))
+        forced_parity(cfg, 2, 2, 40, skip=("nextf",), flags=flags)
         # advance with the oracle (frontier order is irrelevant to the next level's dist)
         op = ir.parse(cfg["ir"])
         an = A.analyze(op, policy="EXPLICIT")
@@ -99,14 +108,15 @@ def _persistent_grid(prog):
     return bps * nsm
 
 
-def test_c3_full_flag():
+@pytest.mark.parametrize("flags", [7, 7 | 32])
+def test_c3_full_flag(flags):
     import torch
     cb = _cb()
     cfg = configs.c3()
     W, H = cfg["W"], cfg["H"]
     op = ir.parse(cfg["ir"])
-    an = A.analyze(op, policy="EXPLICIT")
-    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT)
+    an = A.analyze(op, policy="EXPLICIT", flags=flags)
+    prog = cb.Program(cfg["ir"], flags=flags, poll_policy=cb.POLL_EXPLICIT)
     grid = _persistent_grid(prog)
     dX = to_dev(cfg["buffers"]["X"])
     dY = torch.zeros(W * H, dtype=torch.int32, device="cuda")

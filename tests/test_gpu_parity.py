@@ -152,6 +152,21 @@ def test_random_programs_prune(seed):
     check(txt, grid, bufs, scheds, flags=23)
 
 
+@pytest.mark.parametrize("seed", range(6))
+def test_random_programs_rank_resume(seed):
+    """Combined preempt + resume ranking (CTXB_RANK_RESUME, NEXT N4) on the GPU."""
+    loop = seed % 3 == 0
+    txt, size = random_program(700 + seed, loop=loop, n_body=10)
+    op = ir.parse(txt)
+    grid = 2
+    nout = op.nv - 1 + op.ns - (1 if loop else 0)
+    bufs = random_buffers(seed, op.block, grid, size, nout)
+    r = np.random.default_rng(seed)
+    nw = grid * op.nwarps
+    scheds = [[r.integers(0, 60, nw).astype(np.uint32), r.integers(0, 20, nw).astype(np.uint32)] for _ in range(4)]
+    check(txt, grid, bufs, scheds, flags=7 | 32 | (16 if seed % 2 else 0))
+
+
 def test_c2_half_prune_small():
     cfg = configs.c2(128, 128, 32, polls="half")
     r = np.random.default_rng(2)
