@@ -77,6 +77,15 @@ extern "C" {
                              by the R-10 key; the paper ranks by preemption
                              latency only and notes re-execution can dominate
                              resuming                          */
+#define CTXB_EXACT   64u  /* exact plan search (NEXT N4, R-19): per
+                             window, the minimum-bytes set of values saved at
+                             preempt whose resume closure (re-execution and
+                             reverting as an order-free fixpoint)
+                             restores every required value, by branch and bound
+                             seeded with the greedy CTXB-R1 plan; a window whose
+                             search exceeds exact_budget nodes (or 48 candidate
+                             values) keeps its greedy plan (counted in
+                             ctxb_program_info_t.exact_truncated)               */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */
@@ -125,6 +134,7 @@ typedef struct {
                            the resume path costs this many context bytes per warp
                            (0 = 512 ~ an HBM round trip x one warp's share of HBM
                            bandwidth when every warp of the chip restores)        */
+  uint32_t exact_budget; /* CTXB_EXACT: branch-and-bound nodes per window (0 = 2^20) */
 } ctxb_options;
 
 typedef struct ctxb_program ctxb_program; /* analysed IR kernel + module; library-owned */
@@ -158,6 +168,14 @@ typedef struct {
   uint32_t n_save_stubs;               /* distinct preemption-routine bodies after
                                           sharing                            */
   uint32_t cubin_bytes;                /* size of the compiled sm_100a cubin         */
+  uint32_t exact_windows;              /* CTXB_EXACT: (site, flashback-point) windows
+                                          searched                                    */
+  uint32_t exact_truncated;            /*   of which the search was cut off (budget or
+                                          > 48 candidates): greedy plan kept          */
+  uint32_t exact_improved;             /*   of which the exact plan saves fewer bytes
+                                          than the greedy CTXB-R1 plan                */
+  uint32_t exact_fallback;             /*   greedy kept although the search completed
+                                          (never expected; a consistency check)       */
   double analyze_ms, codegen_ms, compile_ms;
 } ctxb_program_info_t;
 
@@ -186,7 +204,7 @@ const char* ctxb_version(void);
 
 /* Parse + analyse + generate + compile.  `ir_text` need not be
  * NUL-terminated (`len` bytes are read).  opts == NULL means
- * {CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8}.
+ * {CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0}.
  * Errors: _INVALID_ARG, _PARSE, _ANALYSIS, _NVRTC. */
 int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb_program** out);
 int ctxb_program_destroy(ctxb_program* prog);

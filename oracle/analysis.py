@@ -45,6 +45,7 @@ FLAGS_ALL = 7
 FLAG_DEFER = 8            # CS-Defer on top of the mode's own plans
 FLAG_PRUNE = 16           # demand-driven restore (NEXT N4): restore only what LIVE_IN(c) needs
 FLAG_RANK_RESUME = 32     # combined preempt + resume ranking of flashback-points (NEXT N4)
+FLAG_EXACT = 64           # exact minimum-bytes saved set per window (NEXT N4, oracle/exact.py)
 
 DEFER_INSTR_BYTES = 8     # latency-estimate weight of one deferred instruction, in context bytes
 RESUME_LEVEL_BYTES = 512  # FLAG_RANK_RESUME: one dependent memory round trip, in context bytes
@@ -494,6 +495,9 @@ def plan_window(prog, lv, p, c, backups=(), flags=FLAGS_ALL):
     flashback-point.  With FLAG_RELAXED off the basic condition applies."""
     if not (flags & FLAG_RELAXED):
         return basic_plan(prog, lv, p, c)
+    if flags & FLAG_EXACT:
+        from .exact import exact_plan_window
+        return exact_plan_window(prog, lv, p, c, backups, flags)
     w = _Window(prog, lv, p, c, set(backups) if (flags & FLAG_OSRB) else set(), flags)
     w.sweep()
     if not (flags & FLAG_PRUNE) and not w.feasible():
@@ -680,7 +684,7 @@ def analyze(prog: Program, policy="EVERY_INSTR", mode=MODE_CTXBACK, flags=FLAGS_
             every=8, sites=None, keep_candidates=False, defer_instr_bytes=DEFER_INSTR_BYTES,
             resume_level_bytes=RESUME_LEVEL_BYTES) -> Analysis:
     """Compile-time analysis: per poll site, the chosen plan."""
-    an = _analyze(prog, policy, mode, flags & (FLAGS_ALL | FLAG_PRUNE | FLAG_RANK_RESUME), every, sites,
+    an = _analyze(prog, policy, mode, flags & (FLAGS_ALL | FLAG_PRUNE | FLAG_RANK_RESUME | FLAG_EXACT), every, sites,
                   keep_candidates, (defer_instr_bytes, resume_level_bytes))
     an.flags = flags
     if flags & FLAG_DEFER:
@@ -703,8 +707,9 @@ def _analyze(prog, policy, mode, flags, every, sites, keep_candidates, est=None)
                         live, mode=mode, flags=flags)
     backups = []
     if (flags & FLAG_OSRB) and (flags & FLAG_RELAXED):
-        # R-7 selects backups by the bytes of the R-10 choice, whatever the ranking
-        fb = flags & ~FLAG_RANK_RESUME
+        # R-7 selects backups by the bytes of the greedy R-10 choice, whatever
+        # the ranking or the plan search (R-19)
+        fb = flags & ~(FLAG_RANK_RESUME | FLAG_EXACT)
         base = {c: best_plan(prog, lv, heads, c, (), fb).payload_bytes for c in sites}
         for m in osrb_candidates(prog):
             bb = prog.bb_of(m)

@@ -19,7 +19,8 @@
 namespace ctxb {
 namespace {
 
-constexpr uint32_t F_RELAXED = 1, F_REVERT = 2, F_OSRB = 4, F_DEFER = 8, F_PRUNE = 16, F_RANK_RESUME = 32;
+constexpr uint32_t F_RELAXED = 1, F_REVERT = 2, F_OSRB = 4, F_DEFER = 8, F_PRUNE = 16, F_RANK_RESUME = 32,
+                   F_EXACT = 64;
 constexpr uint32_t VEC_B = 128, SCA_B = 4;
 
 bool is_alu(Op o) {
@@ -529,13 +530,413 @@ Plan basic_plan(const Program& P, const Liveness& L, const DefIndex& D, int p, i
   return pl;
 }
 
+// ---- CTXB_EXACT (NEXT N4 "exact min-bytes plan vs greedy"; R-19) ---
+// The paper's rules as an order-free closure: T = values saved at preempt
+// (CURRENT, OSRB backups, or recovered there by reverting, P:92, P:180,
+// P:265); at resume, re-execute a re-executable j whose operand values are
+// known (R-2, R-4) or revert m = nd(r, d+1) whose inputs are known
+// (P:222-229).  Among the T whose closure holds every required value (R-2:
+// live-out results of W + pass-through live-ins; F_PRUNE: final values of
+// LIVE_IN(c)), pick the minimum of (bytes, |T|, T's candidate indices in value
+// order).  Branch and bound, include-first in value order (so the first of
+// several equal keys found is the lexicographically first), with the greedy
+// plan's key as the initial bound and a node budget; a window whose search
+// runs out of budget keeps its greedy plan (counted as truncated).
+struct ExactCfg {
+  uint32_t budget = 1u << 20;   // search nodes per window
+  uint32_t max_cand = 48;       // relevant candidates beyond which the search is skipped
+  uint32_t windows = 0, truncated = 0, improved = 0, fallback = 0;
+};
+
+class ExactWin {
+ public:
+  ExactWin(const Program& P, const Liveness& L, const DefIndex& D, int p, int c, const std::vector<int>& bk,
+           uint32_t flags)
+      : P(P), L(L), w(P, L, D, p, c, {}, 0), p(p), c(c), flags(flags) {
+    std::set<int> regs;
+    std::set<Val> vals;
+    for (int r = 0; r < P.nregs(); r++)
+      if (L.in[c][r]) regs.insert(r);
+    for (int j = p; j < c; j++) {
+      for (int u : P.ins[j].uses) regs.insert(u);
+      if (P.ins[j].defreg >= 0) {
+        regs.insert(P.ins[j].defreg);
+        vals.insert({P.ins[j].defreg, j});
+      }
+    }
+    for (int r : regs) vals.insert({r, PRE});
+    U.assign(vals.begin(), vals.end());   // canonical order: register id, then PRE, then position
+    for (size_t i = 0; i < U.size(); i++) idx[U[i]] = (int)i;
+    if (flags & F_OSRB)
+      for (int m : bk)
+        if (p <= m && m < c) backups.push_back(m);
+    std::sort(backups.begin(), backups.end());
+    // rules: re-executions (program order), then reverts (value order)
+    for (int j = p; j < c; j++)
+      if (w.reexec_kind(j)) {
+        Rule R;
+        R.out = idx.at({P.ins[j].defreg, j});
+        R.j = j;
+        for (auto& x : w.opvals(j)) R.in.push_back(idx.at(x));
+        xr.push_back(R);
+      }
+    for (size_t i = 0; i < U.size(); i++) {
+      RevertRec rec;
+      if (!revert_rule(U[i], &rec)) continue;
+      Rule R;
+      R.out = (int)i;
+      R.j = rec.m;
+      for (auto& x : rec.inputs) R.in.push_back(idx.at(x));
+      rr.push_back(R);
+      rrec[(int)i] = rec;
+    }
+    for (size_t k = 0; k < xr.size(); k++) xr_of_out[xr[k].out] = (int)k;
+  }
+
+  bool revert_rule(const Val& v, RevertRec* rec) const {
+    if (!(flags & F_REVERT)) return false;
+    int m = w.nd(v.r, v.d == PRE ? p : v.d + 1);
+    if (m < 0) return false;
+    if (!revert_spec(P, P.ins[m], v.r, &rec->kind, &rec->others)) return false;
+    rec->v = v;
+    rec->m = m;
+    rec->inputs = {{v.r, m}};
+    for (auto& o : rec->others)
+      if (o.is_reg()) {
+        int u = regid(P, o);
+        rec->inputs.push_back({u, w.rd(u, m)});
+      }
+    return true;
+  }
+
+  std::vector<int> required() const {
+    std::set<int> req;
+    if (flags & F_PRUNE) {
+      for (int r = 0; r < P.nregs(); r++)
+        if (L.in[c][r]) req.insert(idx.at({r, w.rd(r, c)}));
+    } else {
+      for (int j = p; j < c; j++)
+        if (w.liveout_def(j)) req.insert(idx.at({P.ins[j].defreg, j}));
+      for (int r = 0; r < P.nregs(); r++)
+        if (L.in[c][r] && w.rd(r, c) == PRE) req.insert(idx.at({r, PRE}));
+    }
+    return {req.begin(), req.end()};
+  }
+
+  // Values obtainable at preempt with their first derivation (passes in value order).
+  void preempt_derivations() {
+    der.assign(U.size(), {});
+    for (size_t i = 0; i < U.size(); i++)
+      if (w.is_current(U[i])) der[i] = {SK::C, -1, true};
+    for (int m : backups) {
+      int s = P.ins[m].defreg;
+      int i = idx.at({s, w.rd(s, m)});
+      if (!der[i].present) der[i] = {SK::B, m, true};
+    }
+    bool changed = true;
+    while (changed) {
+      changed = false;
+      for (auto& R : rr) {
+        if (der[R.out].present) continue;
+        bool all = true;
+        for (int x : R.in) all = all && der[x].present;
+        if (all) {
+          der[R.out] = {SK::R, R.j, true};
+          changed = true;
+        }
+      }
+    }
+  }
+
+  // Order-free least fixpoint (for the search): worklist over rule input counters.
+  bool covers(const std::vector<char>& T0, const std::vector<int>& req) {
+    known = T0;
+    std::vector<int> cnt(xr.size() + rr.size());
+    std::vector<int> stack;
+    for (size_t k = 0; k < cnt.size(); k++) {   // counts against T0 only
+      const Rule& R = k < xr.size() ? xr[k] : rr[k - xr.size()];
+      int n = 0;
+      for (int x : R.in) n += !T0[x];
+      cnt[k] = n;
+    }
+    for (size_t k = 0; k < cnt.size(); k++) {
+      const Rule& R = k < xr.size() ? xr[k] : rr[k - xr.size()];
+      if (cnt[k] == 0 && !known[R.out]) {
+        known[R.out] = 1;
+        stack.push_back(R.out);
+      }
+    }
+    while (!stack.empty()) {
+      int v = stack.back();
+      stack.pop_back();
+      for (int k : users[v]) {
+        if (--cnt[k] == 0) {
+          const Rule& R = k < (int)xr.size() ? xr[k] : rr[k - xr.size()];
+          if (!known[R.out]) {
+            known[R.out] = 1;
+            stack.push_back(R.out);
+          }
+        }
+      }
+    }
+    for (int q : req)
+      if (!known[q]) return false;
+    return true;
+  }
+
+  std::vector<int> relevant(const std::vector<int>& req) const {
+    std::vector<char> rel(U.size(), 0);
+    for (int q : req) rel[q] = 1;
+    bool changed = true;
+    while (changed) {
+      changed = false;
+      for (auto* rules : {&xr, &rr})
+        for (auto& R : *rules)
+          if (rel[R.out])
+            for (int x : R.in)
+              if (!rel[x]) rel[x] = 1, changed = true;
+    }
+    std::vector<int> out;
+    for (size_t i = 0; i < U.size(); i++)
+      if (rel[i] && der[i].present) out.push_back((int)i);
+    return out;
+  }
+
+  uint32_t vbytes(int i) const { return P.is_vec(U[i].r) ? VEC_B : SCA_B; }
+
+  void dfs(size_t i, uint32_t bytes) {
+    if (++nodes > cfg->budget) {
+      aborted = true;
+      return;
+    }
+    auto key = std::make_pair(bytes, (uint32_t)Tcur.size());
+    if (covers(Tmask, req)) {
+      if (key < best_key) {
+        best_key = key;
+        bestT = Tcur;
+        found = true;
+      }
+      return;
+    }
+    if (i == cand.size() || aborted) return;
+    if (std::make_pair(bytes + min_rest[i], (uint32_t)Tcur.size() + 1) >= best_key) return;
+    std::vector<char> all = Tmask;   // can the remaining candidates still make it?
+    for (size_t k = i; k < cand.size(); k++) all[cand[k]] = 1;
+    if (!covers(all, req)) return;
+    Tmask[cand[i]] = 1;
+    Tcur.push_back(cand[i]);
+    dfs(i + 1, bytes + vbytes(cand[i]));
+    Tcur.pop_back();
+    Tmask[cand[i]] = 0;
+    if (!aborted) dfs(i + 1, bytes);
+  }
+
+  // Returns the exact plan, or an invalid plan if the search was skipped /
+  // truncated (the caller then keeps the greedy plan).
+  Plan solve(const Plan& greedy, ExactCfg* cfg_) {
+    cfg = cfg_;
+    preempt_derivations();
+    req = required();
+    cand = relevant(req);
+    users.assign(U.size(), {});
+    for (size_t k = 0; k < xr.size() + rr.size(); k++) {
+      const Rule& R = k < xr.size() ? xr[k] : rr[k - xr.size()];
+      for (int x : R.in) users[x].push_back((int)k);
+    }
+    cfg->windows++;
+    // Reductions that cannot change the minimum or its tie-break: a candidate
+    // without which even all the others do not suffice is in every feasible T
+    // (forced; common to all solutions, so the lexicographic order of the rest
+    // decides ties); a candidate derivable from the forced ones is in no
+    // minimal T.
+    std::vector<char> all(U.size(), 0), forced(U.size(), 0);
+    for (int u : cand) all[u] = 1;
+    if (!covers(all, req)) {
+      if (greedy.valid) cfg->fallback++;
+      return Plan{};
+    }
+    uint32_t fbytes = 0;
+    for (int u : cand) {
+      all[u] = 0;
+      if (!covers(all, req)) forced[u] = 1, fbytes += vbytes(u), Tcur.push_back(u);
+      all[u] = 1;
+    }
+    covers(forced, req);
+    std::vector<int> rest;
+    for (int u : cand)
+      if (!forced[u] && !known[u]) rest.push_back(u);
+    cand = rest;
+    if (cand.size() > cfg->max_cand) {
+      cfg->truncated++;
+      return Plan{};
+    }
+    min_rest.assign(cand.size() + 1, UINT32_MAX / 2);
+    for (size_t k = cand.size(); k-- > 0;) min_rest[k] = std::min(min_rest[k + 1], vbytes(cand[k]));
+    // greedy's saved set is feasible here, so its key bounds the minimum
+    best_key = greedy.valid ? std::make_pair(greedy.payload_bytes, (uint32_t)greedy.saved.size() + 1)
+                            : std::make_pair(UINT32_MAX, UINT32_MAX);
+    Tmask = forced;
+    dfs(0, fbytes);
+    if (aborted) {
+      cfg->truncated++;
+      return Plan{};
+    }
+    if (!found) {            // infeasible window (or, never expected, greedy's set not found)
+      if (greedy.valid) cfg->fallback++;
+      return Plan{};
+    }
+    Plan pl = build(bestT);
+    if (greedy.valid && pl.payload_bytes < greedy.payload_bytes) cfg->improved++;
+    return pl;
+  }
+
+  // The plan of a saved set T (same construction as oracle/exact.py).
+  Plan build(const std::vector<int>& T) {
+    std::map<int, Supply> ksup;          // value -> supply (first derivation)
+    std::map<int, char> src;             // saved value -> 'C' | 'B' | 'P'
+    for (int i : T) {
+      const Deriv& d = der[i];
+      src[i] = d.k == SK::C ? 'C' : d.k == SK::B ? 'B' : 'P';
+      ksup[i] = {d.k, d.arg};
+    }
+    std::vector<Event> events;
+    std::map<int, std::vector<Supply>> rx;
+    std::map<int, RevertRec> rev;
+    bool changed = true;
+    while (changed) {
+      changed = false;
+      for (auto& R : xr) {
+        if (rx.count(R.j) || ksup.count(R.out)) continue;
+        bool all = true;
+        for (int x : R.in) all = all && ksup.count(x);
+        if (!all) continue;
+        std::vector<Supply> s;
+        for (int x : R.in) s.push_back(ksup.at(x));
+        rx[R.j] = s;
+        ksup[R.out] = {SK::X, R.j};
+        events.push_back({true, R.j, U[R.out]});
+        changed = true;
+      }
+      for (auto& R : rr) {
+        if (ksup.count(R.out)) continue;
+        bool all = true;
+        for (int x : R.in) all = all && ksup.count(x);
+        if (!all) continue;
+        RevertRec rec = rrec.at(R.out);
+        for (int x : R.in) rec.supplies.push_back(ksup.at(x));
+        rev[R.out] = rec;
+        ksup[R.out] = {SK::R, R.j};
+        events.push_back({false, R.j, U[R.out]});
+        changed = true;
+      }
+    }
+    // demand-driven pruning from the required values (in value order)
+    std::set<int> used_x, used_res, used_pre;
+    std::map<int, char> S;
+    std::function<void(int)> pre = [&](int v) {
+      if (!used_pre.insert(v).second) return;
+      const RevertRec& rec = rrec.at(v);
+      for (auto& x : rec.inputs) {
+        int xi = idx.at(x);
+        if (der[xi].k == SK::R) pre(xi);
+      }
+    };
+    std::function<void(int)> demand = [&](int v) {
+      auto it = src.find(v);
+      if (it != src.end()) {
+        S[v] = it->second;
+        if (it->second == 'P') pre(v);
+        return;
+      }
+      const Supply& s = ksup.at(v);
+      if (s.k == SK::X) {
+        if (used_x.insert(s.arg).second)
+          for (auto& x : w.opvals(s.arg)) demand(idx.at(x));
+      } else if (used_res.insert(v).second) {
+        for (auto& x : rev.at(v).inputs) demand(idx.at(x));
+      }
+    };
+    for (int q : req) demand(q);
+    Plan pl;
+    pl.valid = true;
+    pl.c = c;
+    pl.p = p;
+    pl.kind = 0;
+    for (auto& [i, s] : S) {
+      SavedVal sv{s, U[i], -1};
+      if (s == 'B') sv.bkp_m = der[i].arg;
+      pl.saved.push_back(sv);
+      (P.is_vec(U[i].r) ? pl.n_vec : pl.n_sca)++;
+      pl.payload_bytes += vbytes(i);
+    }
+    // at-preempt chains: inputs supplied by their preempt derivation
+    std::vector<int> prev(used_pre.begin(), used_pre.end());
+    std::stable_sort(prev.begin(), prev.end(), [&](int a, int b) { return rrec.at(a).m > rrec.at(b).m; });
+    for (int v : prev) {
+      RevertRec rec = rrec.at(v);
+      for (auto& x : rec.inputs) {
+        const Deriv& d = der[idx.at(x)];
+        rec.supplies.push_back({d.k, d.k == SK::C ? -1 : d.arg});
+      }
+      pl.pre_reverts.push_back(rec);
+      pl.revert_info[U[v]] = rec;
+    }
+    for (int v : used_res) pl.revert_info[U[v]] = rev.at(v);
+    for (auto& e : events)
+      if ((e.is_x && used_x.count(e.j)) || (!e.is_x && used_res.count(idx.at(e.v)))) pl.schedule.push_back(e);
+    for (int j : used_x) pl.reexec_supply[j] = rx.at(j);
+    for (int r = 0; r < P.nregs(); r++)
+      if (L.in[c][r]) {
+        int d = w.rd(r, c);
+        pl.final_.push_back({r, d == PRE ? Supply{SK::C, -1} : ksup.at(idx.at({r, d}))});
+      }
+    pl.n_rev_pre = (uint32_t)used_pre.size();
+    pl.n_rev_res = (uint32_t)used_res.size();
+    pl.n_reexec = (uint32_t)used_x.size();
+    return pl;
+  }
+
+  struct Rule {
+    int out = -1, j = -1;
+    std::vector<int> in;
+  };
+  const Program& P;
+  const Liveness& L;
+  Window w;
+  int p, c;
+  uint32_t flags;
+  std::vector<Val> U;
+  std::map<Val, int> idx;
+  std::vector<int> backups;
+  std::vector<Rule> xr, rr;
+  std::map<int, RevertRec> rrec;
+  std::map<int, int> xr_of_out;
+  std::vector<Deriv> der;
+  std::vector<std::vector<int>> users;
+  std::vector<char> known, Tmask;
+  std::vector<int> req, cand, Tcur, bestT;
+  std::vector<uint32_t> min_rest;
+  std::pair<uint32_t, uint32_t> best_key;
+  uint64_t nodes = 0;
+  bool aborted = false, found = false;
+  ExactCfg* cfg = nullptr;
+};
+
 Plan window_plan(const Program& P, const Liveness& L, const DefIndex& D, int p, int c, const std::vector<int>& bk,
-                 uint32_t flags) {
+                 uint32_t flags, ExactCfg* ex = nullptr) {
   if (!(flags & F_RELAXED)) return basic_plan(P, L, D, p, c);
-  Window w(P, L, D, p, c, (flags & F_OSRB) ? bk : std::vector<int>{}, flags);
-  w.sweep();
-  if (!(flags & F_PRUNE) && !w.feasible()) return Plan{};
-  return w.plan(0);
+  Plan greedy;
+  {
+    Window w(P, L, D, p, c, (flags & F_OSRB) ? bk : std::vector<int>{}, flags);
+    w.sweep();
+    if ((flags & F_PRUNE) || w.feasible()) greedy = w.plan(0);
+  }
+  if ((flags & F_EXACT) && ex) {
+    ExactWin xw(P, L, D, p, c, bk, flags);
+    Plan pl = xw.solve(greedy, ex);
+    if (pl.valid) return pl;
+  }
+  return greedy;
 }
 
 // CTXB_RANK_RESUME (NEXT N4; the paper ranks by preemption latency only and
@@ -586,11 +987,12 @@ uint64_t resume_estimate(const Program& P, const Plan& pl, uint32_t instr_bytes,
 }
 
 Plan best_plan(const Program& P, const Liveness& L, const DefIndex& D, const std::vector<int>& heads, int c,
-               const std::vector<int>& bk, uint32_t flags, uint32_t instr_bytes = 8, uint32_t level_bytes = 512) {
+               const std::vector<int>& bk, uint32_t flags, uint32_t instr_bytes = 8, uint32_t level_bytes = 512,
+               ExactCfg* ex = nullptr) {
   Plan best;
   std::vector<int64_t> bc;
   for (int p = c; p >= heads[c]; p--) {
-    Plan pl = window_plan(P, L, D, p, c, bk, flags);
+    Plan pl = window_plan(P, L, D, p, c, bk, flags, ex);
     if (!pl.valid) continue;
     std::vector<int64_t> k;
     if (flags & F_RANK_RESUME) k.push_back((int64_t)resume_estimate(P, pl, instr_bytes, level_bytes));
@@ -687,7 +1089,7 @@ Analysis analyze(const Program& P, const Options& opt) {
 
 static Analysis analyze_plans(const Program& P, const Options& opt0) {
   Options opt = opt0;
-  opt.flags &= (7u | F_PRUNE | F_RANK_RESUME);
+  opt.flags &= (7u | F_PRUNE | F_RANK_RESUME | F_EXACT);
   Liveness L = liveness(P);
   DefIndex D(P);
   Analysis A;
@@ -710,8 +1112,9 @@ static Analysis analyze_plans(const Program& P, const Options& opt0) {
   }
   uint32_t fl = opt.flags;
   if ((fl & F_OSRB) && (fl & F_RELAXED)) {
-    // R-7 selects backups by the bytes of the R-10 choice, whatever the ranking
-    uint32_t fb = fl & ~F_RANK_RESUME;
+    // R-7 selects backups by the bytes of the greedy R-10 choice, whatever the
+    // ranking or the plan search (R-19)
+    uint32_t fb = fl & ~(F_RANK_RESUME | F_EXACT);
     std::map<int, uint32_t> base;
     for (int c : A.sites) base[c] = best_plan(P, L, D, A.heads, c, {}, fb).payload_bytes;
     for (int m : osrb_candidates(P)) {
@@ -725,8 +1128,15 @@ static Analysis analyze_plans(const Program& P, const Options& opt0) {
       }
     }
   }
+  ExactCfg ex;
+  if (opt.exact_budget) ex.budget = opt.exact_budget;
   for (int c : A.sites)
-    A.plans.push_back(best_plan(P, L, D, A.heads, c, A.backups, fl, opt.defer_instr_bytes, opt.resume_level_bytes));
+    A.plans.push_back(
+        best_plan(P, L, D, A.heads, c, A.backups, fl, opt.defer_instr_bytes, opt.resume_level_bytes, &ex));
+  A.exact_windows = ex.windows;
+  A.exact_truncated = ex.truncated;
+  A.exact_improved = ex.improved;
+  A.exact_fallback = ex.fallback;
   return A;
 }
 

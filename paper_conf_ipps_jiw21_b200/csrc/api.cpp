@@ -308,14 +308,14 @@ const char* ctxb_version(void) { return "ctxb 0.1 (sm_100a, CTXB-R1)"; }
 int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb_program** out) {
   if (!ir_text || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   *out = nullptr;
-  ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512};
-  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 63 || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
+  ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0};
+  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 127 || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
     return fail(CTXB_E_INVALID_ARG, "bad options");
   std::unique_ptr<ctxb_program> p(new ctxb_program);
   p->opt = Options{o.flags, o.mode, o.poll_policy, o.poll_every ? o.poll_every : 8, o.debug,
                    o.flag_depth ? o.flag_depth : 1, o.min_blocks_per_sm,
                    o.defer_instr_bytes ? o.defer_instr_bytes : 8,
-                   o.resume_level_bytes ? o.resume_level_bytes : 512};
+                   o.resume_level_bytes ? o.resume_level_bytes : 512, o.exact_budget};
   try {
     double t0 = now_ms();
     p->prog = parse_ir(std::string(ir_text, len));
@@ -376,6 +376,10 @@ int ctxb_program_info(const ctxb_program* p, ctxb_program_info_t* o) {
   o->resume_maxnreg = p->cg.resume_maxnreg;
   o->n_save_stubs = p->cg.n_save_stubs;
   o->cubin_bytes = (uint32_t)p->cubin.size();
+  o->exact_windows = p->an.exact_windows;
+  o->exact_truncated = p->an.exact_truncated;
+  o->exact_improved = p->an.exact_improved;
+  o->exact_fallback = p->an.exact_fallback;
   o->analyze_ms = p->t_an;
   o->codegen_ms = p->t_cg;
   o->compile_ms = p->t_cc;

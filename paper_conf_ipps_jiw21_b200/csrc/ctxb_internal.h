@@ -143,6 +143,7 @@ struct Options {
   uint32_t flags = 7, mode = 0, policy = 0, every = 8, debug = 0, flag_depth = 1, min_blocks = 0;
   uint32_t defer_instr_bytes = 8;   // CS-Defer latency-estimate weight per deferred instruction
   uint32_t resume_level_bytes = 512;  // CTXB_RANK_RESUME weight of one dependent memory round trip
+  uint32_t exact_budget = 0;          // CTXB_EXACT search nodes per window (0 = default)
 };
 
 struct Analysis {
@@ -154,6 +155,9 @@ struct Analysis {
   std::vector<Plan> live;                               // LIVE plan per site
   std::vector<int> defer;                               // per site: index of the site it defers to
   uint32_t full_ir_bytes = 0;
+  // CTXB_EXACT: windows searched, truncated (budget / size: greedy plan kept),
+  // strictly improved over greedy, and greedy fallbacks (never expected)
+  uint32_t exact_windows = 0, exact_truncated = 0, exact_improved = 0, exact_fallback = 0;
 };
 
 Analysis analyze(const Program& prog, const Options& opt);

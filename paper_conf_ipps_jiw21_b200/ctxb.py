@@ -14,7 +14,7 @@ import numpy as np
 
 __all__ = [
     "LIB_PATH", "CtxbError", "lib",
-    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
+    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
     "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "EXPORTED_SYMBOLS",
@@ -25,7 +25,7 @@ __all__ = [
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libctxb.so")
 
-RELAXED, REVERT, OSRB, ALL, DEFER, PRUNE, RANK_RESUME = 1, 2, 4, 7, 8, 16, 32
+RELAXED, REVERT, OSRB, ALL, DEFER, PRUNE, RANK_RESUME, EXACT = 1, 2, 4, 7, 8, 16, 32, 64
 MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
 DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1, 2, 4, 8, 16
@@ -52,7 +52,7 @@ class _Opts(C.Structure):
     _fields_ = [("flags", C.c_uint32), ("mode", C.c_uint32), ("poll_policy", C.c_uint32),
                 ("poll_every", C.c_uint32), ("debug", C.c_uint32), ("flag_depth", C.c_uint32),
                 ("min_blocks_per_sm", C.c_uint32), ("defer_instr_bytes", C.c_uint32),
-                ("resume_level_bytes", C.c_uint32)]
+                ("resume_level_bytes", C.c_uint32), ("exact_budget", C.c_uint32)]
 
 
 class _SiteInfo(C.Structure):
@@ -65,7 +65,8 @@ class _ProgInfo(C.Structure):
     _fields_ = [(n, C.c_uint32) for n in ("n_instrs", "nv", "ns", "block", "n_buffers", "n_uniforms", "n_sites",
                                           "n_backups", "max_payload_bytes_per_warp", "full_ir_bytes_per_warp",
                                           "num_regs", "compiled", "num_regs_resume", "resume_maxnreg",
-                                          "n_save_stubs", "cubin_bytes")] + \
+                                          "n_save_stubs", "cubin_bytes", "exact_windows", "exact_truncated",
+                                          "exact_improved", "exact_fallback")] + \
                [("analyze_ms", C.c_double), ("codegen_ms", C.c_double), ("compile_ms", C.c_double)]
 
 
@@ -154,9 +155,9 @@ def _u32arr(vals):
 
 def ctxb_analyze(ir_text: str, flags=ALL, mode=MODE_CTXBACK, poll_policy=POLL_EVERY_INSTR, poll_every=8,
                  debug=0, flag_depth=1, min_blocks_per_sm=0, defer_instr_bytes=8,
-                 resume_level_bytes=512) -> "Program":
+                 resume_level_bytes=512, exact_budget=0) -> "Program":
     return Program(ir_text, flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm,
-                   defer_instr_bytes, resume_level_bytes)
+                   defer_instr_bytes, resume_level_bytes, exact_budget)
 
 
 def ctxb_launch(prog, grid, buffers, uniforms, ctx, stream=None, forced=None) -> "Run":
@@ -191,10 +192,11 @@ class Program:
     """An analysed + compiled IR kernel (ctxb_analyze)."""
 
     def __init__(self, ir_text, flags=ALL, mode=MODE_CTXBACK, poll_policy=POLL_EVERY_INSTR, poll_every=8,
-                 debug=0, flag_depth=1, min_blocks_per_sm=0, defer_instr_bytes=8, resume_level_bytes=512):
+                 debug=0, flag_depth=1, min_blocks_per_sm=0, defer_instr_bytes=8, resume_level_bytes=512,
+                 exact_budget=0):
         self._h = C.c_void_p()
         o = _Opts(flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm, defer_instr_bytes,
-                  resume_level_bytes)
+                  resume_level_bytes, exact_budget)
         b = ir_text.encode()
         _chk(lib.ctxb_analyze(b, len(b), C.byref(o), C.byref(self._h)))
         self.debug = debug

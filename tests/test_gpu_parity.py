@@ -185,3 +185,36 @@ def test_smem_barrier_kernel_block_uniform():
     scheds = [[[k] * 6] for k in range(3)] + [[r.integers(0, 3, 6).astype(np.uint32),
                                                r.integers(0, 2, 6).astype(np.uint32)] for _ in range(6)]
     check(SMEM_K, 3, bufs, scheds)
+
+
+@pytest.mark.parametrize("seed", [815, 832, 850, 867, 953, 997])
+def test_random_programs_exact(seed):
+    """Exact minimum-bytes plans (CTXB_EXACT, NEXT N4) on the GPU vs the oracle;
+    the seeds are programs where the exact plan beats greedy at >= 1 site."""
+    loop = seed % 3 == 0
+    txt, size = random_program(seed, loop=loop, n_body=10)
+    op = ir.parse(txt)
+    grid = 2
+    nout = op.nv - 1 + op.ns - (1 if loop else 0)
+    bufs = random_buffers(seed, op.block, grid, size, nout)
+    r = np.random.default_rng(seed)
+    nw = grid * op.nwarps
+    n = len(op.instrs)
+    scheds = [[[k] * nw] for k in range(0, n, 3)] + \
+             [[r.integers(0, 60, nw).astype(np.uint32), r.integers(0, 20, nw).astype(np.uint32)] for _ in range(4)]
+    check(txt, grid, bufs, scheds, flags=7 | 64 | (16 if seed % 2 else 0))
+
+
+@pytest.mark.parametrize("k", [0, 1])
+def test_exact_fixtures_and_c1_on_gpu(k):
+    import json
+    import os
+    if k == 0:
+        cfg = configs.c1()
+        check(cfg["ir"], 1, cfg["buffers"], [[[s] * 4] for s in range(24)], flags=7 | 64)
+    for case in json.load(open(os.path.join(os.path.dirname(__file__), "golden", "exact.json")))["cases"]:
+        op = ir.parse(case["ir"])
+        r = np.random.default_rng(5 + k)
+        bufs = {b: (r.integers(0, 1 << 32, 64, dtype=np.uint64).astype(np.uint32) if kd == "ro"
+                    else np.zeros(64, np.uint32)) for b, kd in op.buffers.items()}
+        check(case["ir"], 1, bufs, [[[s]] for s in range(len(op.instrs))], flags=7 | 64)   # 1 block: outputs indexed by %tid
