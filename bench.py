@@ -163,12 +163,13 @@ class Clocks:
 
 # ---- the GPU arm --------------------------------------------------------------
 
-def make_c2(cb, size, mode, debug=0):
+def make_c2(cb, size, mode, debug=0, flags=None):
     """C2 with one poll site per k-loop iteration (its window spans the whole
     unrolled iteration) and 2 resident blocks / SM (__launch_bounds__)."""
     from workloads import configs
     ir_text = configs.c2_ir(size, size, size, polls="iter")
-    return cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, mode=mode, debug=debug, min_blocks_per_sm=2)
+    return cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, mode=mode, debug=debug, min_blocks_per_sm=2,
+                      flags=cb.ALL if flags is None else flags)
 
 
 def spin_until(t):
@@ -381,7 +382,8 @@ def oracle_sample(steps=1, seed=0):
 
 MODES = (("ctxback", 0, 7), ("full_hw", 3, 7), ("live", 1, 7),
          ("cs_defer", 1, 15), ("ctxback_cs_defer", 0, 15),      # (name, mode, flags); 15 = ALL | DEFER
-         ("ctxback_rank_resume", 0, 39))                        # 39 = ALL | RANK_RESUME (NEXT N4)
+         ("ctxback_rank_resume", 0, 39),                        # 39 = ALL | RANK_RESUME (NEXT N4)
+         ("ctxback_gather", 0, 135), ("full_hw_gather", 3, 135))  # 135 = ALL | GATHER_RESUME
 
 
 def _progs(cb, ir_text, debug=0, min_blocks=0):
@@ -444,8 +446,8 @@ def _flag_trials(progs, grid, make_bufs, uniforms, check, fracs, T_s):
     return out
 
 
-def _reduction(res, name="ctxback"):
-    c, f = res.get(name, {}), res.get("full_hw", {})
+def _reduction(res, name="ctxback", base="full_hw"):
+    c, f = res.get(name, {}), res.get(base, {})
 
     def pct(k):
         if c.get(k) and f.get(k):
@@ -495,6 +497,7 @@ def bench_c1(cb):
             res["static"] = _static(prog, 4)
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
+    res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
     res["cs_defer_reduction_vs_full_hw"] = _reduction(res, "cs_defer")
     res["ctxback_cs_defer_reduction_vs_full_hw"] = _reduction(res, "ctxback_cs_defer")
     res["workload"] = "C1 24-instruction IR kernel, 1 TB x 128 threads, all warps preempted at each of the 24 sites"
@@ -529,6 +532,7 @@ def bench_c2s(cb, trials, seed):
     res["static"]["smem_bytes_per_tb"] = 4 * 2048
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
+    res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
     res["t_uninterrupted_ms"] = round(T, 3)
     res["grid"] = grid
     res["workload"] = ("C2s SGEMM IR 4096^3 with shared-memory k-tiles (8 KiB / TB) and 2 barriers per k-tile; "
@@ -561,6 +565,7 @@ def bench_c3(cb, trials, seed):
     res["static"] = _static(progs["ctxback"], 8)
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
+    res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
     res["cs_defer_reduction_vs_full_hw"] = _reduction(res, "cs_defer")
     res["ctxback_cs_defer_reduction_vs_full_hw"] = _reduction(res, "ctxback_cs_defer")
     res["t_uninterrupted_ms"] = round(T, 3)
@@ -601,6 +606,7 @@ def bench_c4a(cb, trials, seed):
         8 * osrb_off.site_info(k)["payload_bytes_per_warp"] for k in range(osrb_off.num_sites)]
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
+    res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
     res["t_uninterrupted_ms"] = round(T, 3)
     res["grid"] = grid
     res["uninterrupted_equals_bincount"] = ok
@@ -669,6 +675,7 @@ def bench_c4b(cb, trials, seed):
     res["static"] = _static(progs["ctxback"], 8)
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
+    res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
     res["grid"] = grid
     res["largest_level"] = big
     res["workload"] = (f"C4b level-synchronous BFS IR, n=2^22, {len(ci)} edges (Poisson(16) out-degree), "
@@ -937,10 +944,14 @@ def oracle_throughput(max_cores=None):
     t1 = _oracle_tb((0, blob))
     n = max_cores or os.cpu_count() or 1
     ctx = mpr.get_context("fork")
+    import gc
+    gc.collect()
+    gc.freeze()          # forked workers must not collect (and destroy) the parent's library handles
     t0 = time.perf_counter()
     with ctx.Pool(n) as pool:
         pool.map(_oracle_tb, [(b % 16, blob) for b in range(max(n, 16))])
     tw = time.perf_counter() - t0
+    gc.unfreeze()
     model = platform.processor() or ""
     try:
         for line in open("/proc/cpuinfo"):
@@ -971,6 +982,9 @@ def gpu_arm(args):
         progs["live"] = make_c2(cb, size, cb.MODE_LIVE)
         progs["full_hw"] = make_c2(cb, size, cb.MODE_FULL_HW)
         progs["full_ir"] = make_c2(cb, size, cb.MODE_FULL)
+        # CTXB_GATHER_RESUME: resumed warps wait until every preempted warp has restored
+        progs["ctxback_gather"] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | cb.GATHER_RESUME)
+        progs["full_hw_gather"] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | cb.GATHER_RESUME)
     bps, nsm = progs["ctxback"].occupancy()
     for p in progs.values():
         bps = min(bps, p.occupancy()[0])
@@ -1005,7 +1019,7 @@ def gpu_arm(args):
     main = summarize(recs)
     # ---- baselines in the same framework (same fracs) ----
     base = {}
-    for k in ("full_hw", "full_ir", "live"):
+    for k in ("full_hw", "full_ir", "live", "ctxback_gather", "full_hw_gather"):
         if k in progs:
             preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_w[:1], ws)
             r = preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_t, ws)

@@ -87,6 +87,14 @@ extern "C" {
                              values) keeps its greedy plan (counted in
                              ctxb_program_info_t.exact_truncated)               */
 
+#define CTXB_GATHER_RESUME 128u /* runtime: in a resume launch of a persistent grid
+                             (every block resident), a warp that has restored its
+                             context waits until every preempted warp of the
+                             launch has restored (or the flag rises again, or
+                             20 us pass) before continuing, so early warps' work
+                             does not queue the late warps' restores in the
+                             memory system; off: each warp continues at once   */
+
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */
 #define CTXB_MODE_FULL    2u /* save every declared IR register (FULL_IR)        */

@@ -103,6 +103,7 @@ struct ctxb_run {
   CUstream stream = nullptr;
   CUdeviceptr flag = 0, stamps = 0, forced = 0;
   uint32_t epoch = 0;
+  uint32_t rb_target = 0;   // CTXB_GATHER_RESUME: blocks with preempted warps the resume launch waits for
   int state = RUN_RUNNING;
   std::vector<uint32_t> hdr_prev, hdr;  // host header snapshots (launch e-1, e)
   bool resumed_launch = false;
@@ -223,7 +224,7 @@ int compile(ctxb_program* p) {
 void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>& blob) {
   size_t nb = std::max<size_t>(1, p->prog.buf_names.size());
   size_t nu = std::max<size_t>(1, p->prog.uniforms.size());
-  size_t words = nb + 5 + (nu + 6 + 1) / 2;
+  size_t words = nb + 5 + (nu + 8 + 1) / 2;
   blob.assign(words, 0);
   for (size_t i = 0; i < r->bufs.size(); i++) blob[i] = r->bufs[i];
   blob[nb + 0] = r->cbuf;
@@ -239,6 +240,12 @@ void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>
   u[nu + 3] = p->full_hw_bytes();
   u[nu + 4] = 0;   // `zero`: opaque 0 for the timing dependency (gtimer_after)
   u[nu + 5] = p->smem_off();
+  u[nu + 6] = r->resumed_launch ? r->rb_target : 0u;
+  static const uint32_t gather_timeout = [] {   // ns; bounds the wait if a block is not resident
+    const char* e = getenv("CTXB_GATHER_TIMEOUT_NS");
+    return e ? (uint32_t)strtoul(e, nullptr, 10) : 20000u;
+  }();
+  u[nu + 7] = gather_timeout;
 }
 
 int upload_forced(ctxb_run* r, const uint32_t* targets) {
@@ -257,6 +264,7 @@ int upload_forced(ctxb_run* r, const uint32_t* targets) {
 
 int launch(ctxb_run* r, bool resume) {
   std::vector<uint64_t> blob;
+  r->resumed_launch = resume;
   pack_params(r, r->prog, blob);
   void* args[] = {blob.data()};
   Driver& d = driver();
@@ -309,7 +317,7 @@ int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb
   if (!ir_text || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   *out = nullptr;
   ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0};
-  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 127 || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
+  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 255 || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
     return fail(CTXB_E_INVALID_ARG, "bad options");
   std::unique_ptr<ctxb_program> p(new ctxb_program);
   p->opt = Options{o.flags, o.mode, o.poll_policy, o.poll_every ? o.poll_every : 8, o.debug,
@@ -504,7 +512,8 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
   }
   if (!r->flag) {
     CUdeviceptr f = 0, s = 0, t = 0;
-    CU(d.cuMemAlloc(&f, 256));
+    // flag (+0), gather arrivals (+128), a gather release word per block (+256)
+    CU(d.cuMemAlloc(&f, 256 + (size_t)grid * 4));
     CU(d.cuMemAlloc(&s, (size_t)r->n_warps * 32));
     CU(d.cuMemAlloc(&t, (size_t)r->n_warps * 4));
     r->flag = f;
@@ -513,8 +522,8 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
     CU(d.cuEventCreate(&r->ev0, CU_EVENT_DEFAULT));
     CU(d.cuEventCreate(&r->ev1, CU_EVENT_DEFAULT));
     CU(d.cuEventCreate(&r->evf, CU_EVENT_DEFAULT));
-    std::vector<uint32_t> z(64, 0);
-    CU(d.cuMemcpyHtoD(r->flag, z.data(), 256));   // the flag is 0 whenever a run does not hold it raised
+    std::vector<uint32_t> z(64 + grid, 0);
+    CU(d.cuMemcpyHtoD(r->flag, z.data(), z.size() * 4));   // the flag is 0 whenever a run does not hold it raised
   }
   // No header memset: every warp of launch 0 writes its header (DONE or
   // PREEMPTED with epoch 1) before the launch completes.
@@ -579,6 +588,28 @@ int ctxb_resume(ctxb_run* r, void* stream, const uint32_t* forced_targets) {
   r->stream = (CUstream)stream;
   int rc = upload_forced(r, forced_targets);
   if (rc) return rc;
+  r->rb_target = 0;
+  if (r->prog->opt.flags & CTXB_GATHER_RESUME) {
+    // wait only for warps that can all be resident at once (persistent grid)
+    Driver& d = driver();
+    int b = 0, n = 0;
+    CUdevice dev;
+    CU(d.cuOccupancyMaxActiveBlocksPerMultiprocessor(&b, r->mod.resume, r->prog->prog.block, 0));
+    CU(d.cuCtxGetDevice(&dev));
+    CU(d.cuDeviceGetAttribute(&n, CU_DEVICE_ATTRIBUTE_MULTIPROCESSOR_COUNT, dev));
+    if ((uint64_t)r->grid <= (uint64_t)b * (uint64_t)n) {
+      // target = blocks with >= 1 preempted warp (one global arrival per block)
+      uint32_t nwb = r->prog->prog.block / 32, blocks = 0;
+      for (uint32_t b = 0; b < r->grid; b++) {
+        bool any = false;
+        for (uint32_t w = b * nwb; w < (b + 1) * nwb; w++)
+          any = any || (r->hdr[(size_t)w * 4 + 2] == CTXB_STATE_PREEMPTED && r->hdr[(size_t)w * 4 + 3] == r->epoch);
+        blocks += any;
+      }
+      r->rb_target = blocks;
+      CU(d.cuMemsetD32Async(r->flag + 128, 0, 32 + r->grid, r->stream));   // arrivals + release words
+    }
+  }
   r->epoch++;
   return launch(r, true);
 }

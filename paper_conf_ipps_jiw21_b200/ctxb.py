@@ -14,7 +14,7 @@ import numpy as np
 
 __all__ = [
     "LIB_PATH", "CtxbError", "lib",
-    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
+    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "GATHER_RESUME", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
     "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "EXPORTED_SYMBOLS",
@@ -25,7 +25,7 @@ __all__ = [
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libctxb.so")
 
-RELAXED, REVERT, OSRB, ALL, DEFER, PRUNE, RANK_RESUME, EXACT = 1, 2, 4, 7, 8, 16, 32, 64
+RELAXED, REVERT, OSRB, ALL, DEFER, PRUNE, RANK_RESUME, EXACT, GATHER_RESUME = 1, 2, 4, 7, 8, 16, 32, 64, 128
 MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
 DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1, 2, 4, 8, 16
@@ -195,6 +195,7 @@ class Program:
                  debug=0, flag_depth=1, min_blocks_per_sm=0, defer_instr_bytes=8, resume_level_bytes=512,
                  exact_budget=0):
         self._h = C.c_void_p()
+        self._pid = os.getpid()
         o = _Opts(flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm, defer_instr_bytes,
                   resume_level_bytes, exact_budget)
         b = ir_text.encode()
@@ -202,7 +203,8 @@ class Program:
         self.debug = debug
 
     def __del__(self):
-        if getattr(self, "_h", None):
+        # a forked child (e.g. a multiprocessing worker) does not own the handle
+        if getattr(self, "_h", None) and getattr(self, "_pid", None) == os.getpid():
             lib.ctxb_program_destroy(self._h)
             self._h = None
 
@@ -275,12 +277,13 @@ class Run:
 
     def __init__(self, h, prog, grid, keep):
         self._h = h
+        self._pid = os.getpid()
         self.prog = prog
         self.grid = grid
         self._keep = keep          # keep the caller's tensors alive
 
     def __del__(self):
-        if getattr(self, "_h", None):
+        if getattr(self, "_h", None) and getattr(self, "_pid", None) == os.getpid():
             lib.ctxb_run_destroy(self._h)
             self._h = None
 

@@ -75,6 +75,18 @@ def test_c4a_small_forced():
     assert an.backups, "C4a must select an OSRB backup"
 
 
+def test_c4a_small_forced_gather():
+    """CTXB_GATHER_RESUME (resumed warps wait until every preempted warp of
+    the launch has restored): outputs and headers unchanged, nested."""
+    cfg = configs.c4a(1 << 14, grid=2)
+    forced_parity(cfg, 2, 3, 4, flags=7 | 128)
+
+
+def test_c3_small_forced_gather():
+    cfg = configs.c3(512, 128, 64)
+    forced_parity(cfg, 4, 3, 128, flags=7 | 128)
+
+
 @pytest.mark.parametrize("flags", [7, 7 | 32])
 def test_c4b_small_forced_level(flags):
     rp, ci = configs.c4b_graph(1 << 10, 16)
@@ -141,14 +153,14 @@ def test_c3_full_flag(flags):
     assert npre > 0
 
 
-@pytest.mark.parametrize("skewed", [False, True])
-def test_c4a_full_flag(skewed):
+@pytest.mark.parametrize("skewed,gather", [(False, 0), (True, 0), (False, 128)])
+def test_c4a_full_flag(skewed, gather):
     import torch
     cb = _cb()
     cfg = configs.c4a(1 << 28, skewed=skewed, grid=1)
     op = ir.parse(cfg["ir"])
     an = A.analyze(op, policy="EXPLICIT")
-    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT)
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | gather)
     assert prog.backups == an.backups and prog.backups
     grid = _persistent_grid(prog)
     keys = cfg["buffers"]["keys"]

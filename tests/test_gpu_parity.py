@@ -218,3 +218,11 @@ def test_exact_fixtures_and_c1_on_gpu(k):
         bufs = {b: (r.integers(0, 1 << 32, 64, dtype=np.uint64).astype(np.uint32) if kd == "ro"
                     else np.zeros(64, np.uint32)) for b, kd in op.buffers.items()}
         check(case["ir"], 1, bufs, [[[s]] for s in range(len(op.instrs))], flags=7 | 64)   # 1 block: outputs indexed by %tid
+
+
+def test_c1_gather_resume_nested():
+    """CTXB_GATHER_RESUME with forced nested preemption and poison (C1)."""
+    cfg = configs.c1()
+    vecs = configs.c1_random_site_vectors(64, seed=11)
+    scheds = [[[k] * 4] for k in range(0, 24, 2)] + [[v, v // 2] for v in vecs[:32]]
+    check(cfg["ir"], 1, cfg["buffers"], scheds, flags=7 | 128)

@@ -12,6 +12,7 @@ import paper_conf_ipps_jiw21_b200 as cb  # noqa: E402
 from workloads import configs  # noqa: E402
 
 which = sys.argv[1] if len(sys.argv) > 1 else "c3"
+gather = cb.GATHER_RESUME if "gather" in sys.argv[2:] else 0
 if which == "c3":
     cfg = configs.c3()
     mk = lambda: [torch.from_numpy(cfg["buffers"]["X"].view(np.int32)).cuda(),  # noqa: E731
@@ -32,7 +33,7 @@ else:
 bufs = mk()
 s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
 for name, mode in (("ctxback", 0), ("full_hw", 3), ("full_ir", 2), ("live", 1)):
-    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, mode=mode, min_blocks_per_sm=mb)
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, mode=mode, min_blocks_per_sm=mb, flags=cb.ALL | gather)
     bps, nsm = prog.occupancy()
     grid = bps * nsm
     ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
@@ -54,7 +55,7 @@ for name, mode in (("ctxback", 0), ("full_hw", 3), ("full_ir", 2), ("live", 1)):
         ms = run.launch_ms()
         stp = run.stamps()[pre]
         ent, site = stp[:, 2].astype(np.int64), stp[:, 3].astype(np.int64)
-        if which == "c4a":
+        if which in ("c4a", "c4b") or gather:
             order = np.argsort(ent)
             print("   entry quantiles (us from first):", np.percentile((ent - ent.min()) / 1e3, [0, 50, 90, 99, 100]).round(2),
                   "site quantiles:", np.percentile((site - ent.min()) / 1e3, [0, 50, 90, 99, 100]).round(2),
