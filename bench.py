@@ -315,8 +315,8 @@ def poll_overhead(cb, size, grid, bufs, reps=20):
 
 def one_direction_peaks(gib=2, reps=5):
     """Reference for the save (write-only) and restore (read-only) kernels:
-    the best of `reps` torch fill_ (writes) and sum (reads, int64 accumulate)
-    over a `gib` GiB int32 buffer, CUDA events.  MEASURED_PEAKS.json's copy
+    the best of `reps` torch fill_ (writes) and float32 sum (reads) over a
+    `gib` GiB buffer, CUDA events.  MEASURED_PEAKS.json's copy
     figure counts read + write bytes, which a one-direction stream can beat."""
     import torch
     buf = torch.empty(gib << 28, dtype=torch.int32, device="cuda")
@@ -329,15 +329,16 @@ def one_direction_peaks(gib=2, reps=5):
         e1.record()
         torch.cuda.synchronize()
         best_w = max(best_w, nbytes / (e0.elapsed_time(e1) * 1e6))
+    fbuf = buf.view(torch.float32)
     for _ in range(reps):
         e0.record()
-        buf.sum(dtype=torch.int64)
+        fbuf.sum()
         e1.record()
         torch.cuda.synchronize()
         best_r = max(best_r, nbytes / (e0.elapsed_time(e1) * 1e6))
     del buf
     return {"write_only_gbs": round(best_w, 1), "read_only_gbs": round(best_r, 1),
-            "how": f"torch fill_ / sum over {gib} GiB int32, best of {reps}, CUDA events (live, this run)"}
+            "how": f"torch fill_ (write) / float32 sum (read) over {gib} GiB, best of {reps}, CUDA events (live, this run)"}
 
 
 def peaks():
@@ -413,9 +414,9 @@ MODES = (("ctxback", 0, 7), ("full_hw", 3, 7), ("live", 1, 7),
          ("ctxback_gather", 0, 135), ("full_hw_gather", 3, 135))  # 135 = ALL | GATHER_RESUME
 
 
-def _progs(cb, ir_text, debug=0, min_blocks=0):
+def _progs(cb, ir_text, debug=0, min_blocks=0, extra_flags=0):
     return {name: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT if "poll" in ir_text else cb.POLL_EVERY_INSTR,
-                             mode=mode, flags=flags, debug=debug, min_blocks_per_sm=min_blocks)
+                             mode=mode, flags=flags | extra_flags, debug=debug, min_blocks_per_sm=min_blocks)
             for name, mode, flags in MODES}
 
 
@@ -606,7 +607,8 @@ def bench_c4a(cb, trials, seed):
     import torch
     from workloads import configs
     cfg = configs.c4a(1 << 28, grid=1)
-    progs = _progs(cb, cfg["ir"])
+    # one poll per ~6 us chunk: sites test the flag they load (CTXB_SYNC_POLL), in every mode
+    progs = _progs(cb, cfg["ir"], extra_flags=cb.SYNC_POLL)
     grid = _grid(progs)
     keys = cfg["buffers"]["keys"]
     want = torch.from_numpy(np.bincount(keys >> 24, minlength=256).astype(np.int32)).cuda()
@@ -638,7 +640,7 @@ def bench_c4a(cb, trials, seed):
     res["grid"] = grid
     res["uninterrupted_equals_bincount"] = ok
     res["workload"] = ("C4a 256-bin histogram IR, 2^28 uniform u32 keys (1 GiB), global atomics into per-block "
-                       "bin copies, flag at U[0.05,0.95] x T")
+                       "bin copies, flag at U[0.05,0.95] x T; every mode compiled with CTXB_SYNC_POLL")
     return res
 
 

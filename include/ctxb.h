@@ -95,6 +95,12 @@ extern "C" {
                              does not queue the late warps' restores in the
                              memory system; off: each warp continues at once   */
 
+#define CTXB_SYNC_POLL   256u /* codegen: a poll site tests the flag value it loads
+                             itself (one L2 round trip per poll) instead of the
+                             value loaded flag_depth sites earlier: detection
+                             within one site interval instead of flag_depth + 1,
+                             for loops whose iterations are long (C4a)         */
+
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */
 #define CTXB_MODE_FULL    2u /* save every declared IR register (FULL_IR)        */

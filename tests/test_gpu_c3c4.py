@@ -153,7 +153,7 @@ def test_c3_full_flag(flags):
     assert npre > 0
 
 
-@pytest.mark.parametrize("skewed,gather", [(False, 0), (True, 0), (False, 128)])
+@pytest.mark.parametrize("skewed,gather", [(False, 0), (True, 0), (False, 128), (True, 256), (False, 384)])
 def test_c4a_full_flag(skewed, gather):
     import torch
     cb = _cb()
