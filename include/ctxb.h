@@ -91,9 +91,10 @@ extern "C" {
                              (every block resident), a warp that has restored its
                              context waits until every preempted warp of the
                              launch has restored (or the flag rises again, or
-                             20 us pass) before continuing, so early warps' work
-                             does not queue the late warps' restores in the
-                             memory system; off: each warp continues at once   */
+                             20 us pass; env CTXB_GATHER_TIMEOUT_NS) before
+                             continuing, so early warps' work does not queue the
+                             late warps' restores in the memory system; off:
+                             each warp continues at once                        */
 
 #define CTXB_SYNC_POLL   256u /* codegen: a poll site tests the flag value it loads
                              itself (one L2 round trip per poll) instead of the

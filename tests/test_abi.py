@@ -110,3 +110,18 @@ def test_context_capacity_layout():
     for grid in (1, 7, 148):
         nw = grid * 4
         assert p.context_capacity(grid) == ((nw * 16 + 255) // 256) * 256 + nw * max(128, stride)
+
+
+def test_runtime_options_generate_and_compile():
+    """CTXB_GATHER_RESUME and CTXB_SYNC_POLL change only the generated code
+    (plans identical); both compile for sm_100a with NVRTC."""
+    from workloads import configs
+    txt = configs.c4a_ir(1 << 14)
+    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
+    g = cb.Program(txt, flags=cb.ALL | cb.GATHER_RESUME | cb.SYNC_POLL, poll_policy=cb.POLL_EXPLICIT)
+    assert g.info["compiled"] == 1
+    assert [g.plan_text(k) for k in range(g.num_sites)] == [base.plan_text(k) for k in range(base.num_sites)]
+    src = g.source
+    assert "resume_gather(P, lane, cta, dep" in src and "bar.sync 1" in src
+    assert "__any_sync(0xffffffffu, ld_flag(flagp) != 0u)" in src
+    assert "resume_gather(P" not in base.source and "ld_flag(flagp) != 0u)" not in base.source
