@@ -101,6 +101,20 @@ extern "C" {
                              value loaded flag_depth sites earlier: detection
                              within one site interval instead of flag_depth + 1,
                              for loops whose iterations are long (C4a)         */
+#define CTXB_HOST_SIGNAL 512u /* runtime + codegen: ctxb_preempt also raises a word
+                             in mapped pinned host memory.  Each warp reads it
+                             (system-scope load over PCIe, tested one site
+                             later) once every ceil(n_warps / R) of its polls,
+                             staggered by warp id (R = env CTXB_HOST_RELAYS,
+                             default 1: ~R reads per poll interval device-wide)
+                             and forwards a raised word to the device flag
+                             that every warp polls; the stream memory op is
+                             still issued as the fallback (env
+                             CTXB_HOST_SIGNAL_ONLY=1 drops it: tests).  Cuts the signal's
+                             ~7.6 us stream-memop path.  Flag
+                             mode only (ignored by CTXB_DEBUG_FORCED).
+                             stats.signal_to_drained_us is 0 in this mode (the
+                             host store is not stream-ordered): use host_us   */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */

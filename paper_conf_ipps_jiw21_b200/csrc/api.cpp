@@ -1,6 +1,7 @@
 // C ABI of libctxb (include/ctxb.h).  Compile-time part: P:311-317; runtime
 // part: P:319-323 (preemption), P:313-315 (resume).
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cstring>
 #include <map>
@@ -62,6 +63,8 @@ struct ctxb_program {
     CUdeviceptr flag = 0, stamps = 0, forced = 0;
     uint32_t n_warps = 0;
     CUevent ev0 = nullptr, ev1 = nullptr, evf = nullptr;
+    void* hflag = nullptr;    // CTXB_HOST_SIGNAL: mapped pinned host word (else NULL)
+    CUdeviceptr hflag_dev = 0;
   };
   std::vector<Res> pool;   // per-run device resources, reused (flag is always left at 0)
   uint32_t full_ir_words128() const {  // 128-B rows occupied by the FULL_IR layout
@@ -102,6 +105,8 @@ struct ctxb_run {
   uint64_t cbytes = 0, pay_off = 0, stride = 0;
   CUstream stream = nullptr;
   CUdeviceptr flag = 0, stamps = 0, forced = 0;
+  void* hflag = nullptr;    // CTXB_HOST_SIGNAL: preemption word in mapped pinned host memory
+  CUdeviceptr hflag_dev = 0;
   uint32_t epoch = 0;
   uint32_t rb_target = 0;   // CTXB_GATHER_RESUME: blocks with preempted warps the resume launch waits for
   int state = RUN_RUNNING;
@@ -112,7 +117,7 @@ struct ctxb_run {
   ~ctxb_run() {
     if (flag && prog) {   // return the resources to the program's pool
       std::lock_guard<std::mutex> g(prog->mu);
-      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf});
+      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf, hflag, hflag_dev});
     }
   }
 };
@@ -224,7 +229,7 @@ int compile(ctxb_program* p) {
 void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>& blob) {
   size_t nb = std::max<size_t>(1, p->prog.buf_names.size());
   size_t nu = std::max<size_t>(1, p->prog.uniforms.size());
-  size_t words = nb + 5 + (nu + 8 + 1) / 2;
+  size_t words = nb + 6 + (nu + 9 + 1) / 2;
   blob.assign(words, 0);
   for (size_t i = 0; i < r->bufs.size(); i++) blob[i] = r->bufs[i];
   blob[nb + 0] = r->cbuf;
@@ -232,7 +237,8 @@ void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>
   blob[nb + 2] = r->forced;
   blob[nb + 3] = r->stamps;
   blob[nb + 4] = r->pay_off;
-  uint32_t* u = reinterpret_cast<uint32_t*>(&blob[nb + 5]);
+  blob[nb + 5] = r->hflag_dev;
+  uint32_t* u = reinterpret_cast<uint32_t*>(&blob[nb + 6]);
   for (size_t i = 0; i < r->uni.size(); i++) u[i] = r->uni[i];
   u[nu + 0] = r->epoch;
   u[nu + 1] = (uint32_t)r->stride;
@@ -246,6 +252,12 @@ void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>
     return e ? (uint32_t)strtoul(e, nullptr, 10) : 20000u;
   }();
   u[nu + 7] = gather_timeout;
+  // CTXB_HOST_SIGNAL: R host-word reads per poll interval device-wide: each
+  // warp reads once every ceil(n_warps / R) of its polls
+  const char* re = getenv("CTXB_HOST_RELAYS");
+  uint32_t relays = re ? (uint32_t)strtoul(re, nullptr, 10) : 1u;
+  relays = relays ? relays : 1u;
+  u[nu + 8] = std::max<uint32_t>(1u, (r->n_warps + relays - 1) / relays);
 }
 
 int upload_forced(ctxb_run* r, const uint32_t* targets) {
@@ -317,7 +329,7 @@ int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb
   if (!ir_text || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   *out = nullptr;
   ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0};
-  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 511 || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
+  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 1023 || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
     return fail(CTXB_E_INVALID_ARG, "bad options");
   std::unique_ptr<ctxb_program> p(new ctxb_program);
   p->opt = Options{o.flags, o.mode, o.poll_policy, o.poll_every ? o.poll_every : 8, o.debug,
@@ -360,6 +372,7 @@ int ctxb_program_destroy(ctxb_program* p) {
       d.cuEventDestroy(r.ev0);
       d.cuEventDestroy(r.ev1);
       d.cuEventDestroy(r.evf);
+      if (r.hflag) d.cuMemFreeHost(r.hflag);
     }
   }
   delete p;
@@ -506,6 +519,8 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
         r->ev0 = p->pool[i].ev0;
         r->ev1 = p->pool[i].ev1;
         r->evf = p->pool[i].evf;
+        r->hflag = p->pool[i].hflag;
+        r->hflag_dev = p->pool[i].hflag_dev;
         p->pool.erase(p->pool.begin() + (long)i);
         break;
       }
@@ -525,6 +540,13 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
     std::vector<uint32_t> z(64 + grid, 0);
     CU(d.cuMemcpyHtoD(r->flag, z.data(), z.size() * 4));   // the flag is 0 whenever a run does not hold it raised
   }
+  if ((p->opt.flags & CTXB_HOST_SIGNAL) && !r->hflag) {
+    void* h = nullptr;
+    CU(d.cuMemHostAlloc(&h, 128, CU_MEMHOSTALLOC_DEVICEMAP | CU_MEMHOSTALLOC_PORTABLE));
+    memset(h, 0, 128);
+    r->hflag = h;
+    CU(d.cuMemHostGetDevicePointer(&r->hflag_dev, h, 0));
+  }
   // No header memset: every warp of launch 0 writes its header (DONE or
   // PREEMPTED with epoch 1) before the launch completes.
   rc = upload_forced(r.get(), forced_targets);
@@ -542,11 +564,23 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
   if ((CUstream)ctrl == r->stream && ctrl != nullptr)
     return fail(CTXB_E_INVALID_ARG, "ctrl_stream must differ from the run's stream");
   Driver& d = driver();
+  volatile uint32_t* hf = static_cast<volatile uint32_t*>(r->hflag);
   double t0 = now_ms();
+  if (hf) {
+    // CTXB_HOST_SIGNAL: relay warps see this store over PCIe and raise the
+    // device flag; the stream memory op below stays as the fallback (every
+    // relay warp may have finished already)
+    *hf = 1u;
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+  }
+  // test knob: CTXB_HOST_SIGNAL_ONLY=1 drops the fallback, so the relay is the only path
+  const char* ho = hf ? getenv("CTXB_HOST_SIGNAL_ONLY") : nullptr;
+  const bool host_only = ho && atoi(ho) != 0;
   CU(d.cuEventRecord(r->evf, (CUstream)ctrl));
-  CU(d.cuStreamWriteValue32((CUstream)ctrl, r->flag, 1u, 0));
+  if (!(hf && host_only)) CU(d.cuStreamWriteValue32((CUstream)ctrl, r->flag, 1u, 0));
   CU(d.cuStreamSynchronize(r->stream));
   double t1 = now_ms();
+  if (hf) *hf = 0u;   // the victim has drained: no warp of this run reads it until the next launch
   CU(d.cuMemsetD32Async(r->flag, 0, 1, (CUstream)ctrl));
   CU(d.cuStreamSynchronize((CUstream)ctrl));
   int rc = collect(r);
@@ -577,7 +611,8 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     CU(d.cuStreamSynchronize((CUstream)ctrl));
     float ms = 0;
     CU(d.cuEventElapsedTime(&ms, r->evf, r->ev1));
-    st->signal_to_drained_us = (double)ms * 1e3;
+    // with CTXB_HOST_SIGNAL the signal is the host store, which the event does not bound
+    st->signal_to_drained_us = hf ? 0.0 : (double)ms * 1e3;
   }
   return CTXB_OK;
 }

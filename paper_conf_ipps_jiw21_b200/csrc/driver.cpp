@@ -52,7 +52,9 @@ Driver& driver() {
               sym(h, "cuEventElapsedTime", &d.cuEventElapsedTime, &e) &&
               sym(h, "cuEventDestroy_v2", &d.cuEventDestroy, &e) && sym(h, "cuEventQuery", &d.cuEventQuery, &e) &&
               sym(h, "cuStreamCreate", &d.cuStreamCreate, &e) && sym(h, "cuStreamDestroy_v2", &d.cuStreamDestroy, &e) &&
-              sym(h, "cuMemcpyDtoHAsync_v2", &d.cuMemcpyDtoHAsync, &e);
+              sym(h, "cuMemcpyDtoHAsync_v2", &d.cuMemcpyDtoHAsync, &e) &&
+              sym(h, "cuMemHostAlloc", &d.cuMemHostAlloc, &e) && sym(h, "cuMemFreeHost", &d.cuMemFreeHost, &e) &&
+              sym(h, "cuMemHostGetDevicePointer_v2", &d.cuMemHostGetDevicePointer, &e);
     if (ok && !sym(h, "cuStreamWriteValue32_v2", &d.cuStreamWriteValue32, &e))
       ok = sym(h, "cuStreamWriteValue32", &d.cuStreamWriteValue32, &e);
     if (!ok) return;

@@ -125,3 +125,24 @@ def test_runtime_options_generate_and_compile():
     assert "resume_gather(P, lane, cta, dep" in src and "bar.sync 1" in src
     assert "__any_sync(0xffffffffu, ld_flag(flagp) != 0u)" in src
     assert "resume_gather(P" not in base.source and "ld_flag(flagp) != 0u)" not in base.source
+
+
+def test_host_signal_generates_and_compiles():
+    """CTXB_HOST_SIGNAL changes only the generated poll sites
+    (plans identical): relay warps load the host word with a system-scope load
+    and forward it; it compiles for sm_100a alone and with CTXB_SYNC_POLL."""
+    from workloads import configs
+    txt = configs.c4a_ir(1 << 14)
+    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
+    for extra in (0, cb.SYNC_POLL):
+        h = cb.Program(txt, flags=cb.ALL | cb.HOST_SIGNAL | extra, poll_policy=cb.POLL_EXPLICIT)
+        assert h.info["compiled"] == 1
+        assert [h.plan_text(k) for k in range(h.num_sites)] == [base.plan_text(k) for k in range(base.num_sites)]
+        src = h.source
+        assert "ld.relaxed.sys.global.u32" in src and "relay_fwd(hfl, flagp, lane) != 0u)" in src
+        assert "hfl = ld_hflag(hflagp); } else hfl = 0u;" in src
+    assert "relay_fwd(hfl" not in base.source
+    # forced (debug) programs ignore the option: no relay code is emitted
+    f = cb.Program(txt, flags=cb.ALL | cb.HOST_SIGNAL, poll_policy=cb.POLL_EXPLICIT,
+                   debug=cb.DEBUG_FORCED | cb.DEBUG_NO_COMPILE)
+    assert "relay_fwd(hfl" not in f.source

@@ -212,12 +212,16 @@ def test_c2s_full_flag_equals_c2():
     assert npre > 0
 
 
-@pytest.mark.parametrize("which", ["c2", "c3", "c2s"])
-def test_flag_mode_repeated_nested_preemption(which):
+@pytest.mark.parametrize("which,host", [("c2", False), ("c3", False), ("c2s", False),
+                                        ("c2", True), ("c3", True), ("c2s", True)])
+def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     """random flag times, repeated and nested
     preempt -> resume -> preempt ... cycles (each resume can be preempted
     again, also inside the same basic-block pass: the LIVE fallback, R-16);
-    the final output stays bit-exact with the uninterrupted run."""
+    the final output stays bit-exact with the uninterrupted run.  host=True:
+    CTXB_HOST_SIGNAL with the stream-memop fallback disabled
+    (CTXB_HOST_SIGNAL_ONLY=1), so every preemption arrives through a relay
+    warp's system-scope poll of the host word."""
     import time
     import torch
     cb = _cb()
@@ -230,7 +234,10 @@ def test_flag_mode_repeated_nested_preemption(which):
         bufs = [to_dev(cfg["buffers"]["A"]), to_dev(cfg["buffers"]["B"]),
                 torch.zeros(4096 * 4096, dtype=torch.int32, device="cuda")]
         out_i, mb = 2, 2
-    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=mb)
+    if host:
+        monkeypatch.setenv("CTXB_HOST_SIGNAL_ONLY", "1")
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=mb,
+                      flags=cb.ALL | (cb.HOST_SIGNAL if host else 0))
     bps, nsm = prog.occupancy()
     grid = bps * nsm
     ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
