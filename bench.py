@@ -482,7 +482,8 @@ def _reduction(res, name="ctxback", base="full_hw"):
             return round(100 * (1 - c[k] / f[k]), 2)
         return None
     return {"latency_pct": pct("latency_us_median"), "signal_to_drained_pct": pct("signal_to_drained_us_median"),
-            "resume_pct": pct("resume_us_median"), "context_pct": pct("context_bytes_per_tb")}
+            "resume_pct": pct("resume_us_median"), "context_pct": pct("context_bytes_per_tb"),
+            "host_latency_pct": pct("host_latency_us_median")}
 
 
 def bench_c1(cb):
@@ -1014,6 +1015,9 @@ def gpu_arm(args):
         # CTXB_GATHER_RESUME: resumed warps wait until every preempted warp has restored
         progs["ctxback_gather"] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | cb.GATHER_RESUME)
         progs["full_hw_gather"] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | cb.GATHER_RESUME)
+        # CTXB_ARMED_SIGNAL: the signal is pre-enqueued at launch behind a host gate
+        progs["ctxback_armed"] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | cb.ARMED_SIGNAL)
+        progs["full_hw_armed"] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | cb.ARMED_SIGNAL)
     bps, nsm = progs["ctxback"].occupancy()
     for p in progs.values():
         bps = min(bps, p.occupancy()[0])
@@ -1048,7 +1052,7 @@ def gpu_arm(args):
     main = summarize(recs)
     # ---- baselines in the same framework (same fracs) ----
     base = {}
-    for k in ("full_hw", "full_ir", "live", "ctxback_gather", "full_hw_gather"):
+    for k in ("full_hw", "full_ir", "live", "ctxback_gather", "full_hw_gather", "ctxback_armed", "full_hw_armed"):
         if k in progs:
             preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_w[:1], ws)
             r = preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_t, ws)
@@ -1167,6 +1171,8 @@ def gpu_arm(args):
             "context_pct": (round(100 * (1 - main["context_bytes_per_tb"] / base["full_hw"]["context_bytes_per_tb"]), 2)
                             if "full_hw" in base and base["full_hw"].get("context_bytes_per_tb") and
                             main.get("context_bytes_per_tb") else None)},
+        "armed_reduction_vs_full_hw_armed": (_reduction(base, "ctxback_armed", "full_hw_armed")
+                                             if "ctxback_armed" in base and "full_hw_armed" in base else None),
         "poll_overhead": ovh, "bulk": bulk, "configs": extra_cfg,
         "roofline": rf, "roofline_restore": rr,
         "cpu_baseline": cpu,

@@ -115,6 +115,18 @@ extern "C" {
                              mode only (ignored by CTXB_DEBUG_FORCED).
                              stats.signal_to_drained_us is 0 in this mode (the
                              host store is not stream-ordered): use host_us   */
+#define CTXB_ARMED_SIGNAL 1024u /* runtime: every launch (and resume) pre-enqueues
+                             its preemption signal on a library-owned
+                             greatest-priority stream: cuStreamWaitValue32 on a
+                             gate word in mapped pinned host memory, then the
+                             signal event and cuStreamWriteValue32(flag).
+                             ctxb_preempt then only stores the gate value (no
+                             driver call on the preemption path; ctrl_stream
+                             is not used); a launch that completes unpreempted
+                             is disarmed when it is collected (ctxb_wait /
+                             ctxb_query / destroy).  Kernels are unchanged.
+                             signal_to_drained_us = signal event (after the
+                             gate opened) -> victim drained    */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */

@@ -63,8 +63,10 @@ struct ctxb_program {
     CUdeviceptr flag = 0, stamps = 0, forced = 0;
     uint32_t n_warps = 0;
     CUevent ev0 = nullptr, ev1 = nullptr, evf = nullptr;
-    void* hflag = nullptr;    // CTXB_HOST_SIGNAL: mapped pinned host word (else NULL)
+    void* hflag = nullptr;    // CTXB_HOST_SIGNAL / CTXB_ARMED_SIGNAL: mapped pinned host words (else NULL)
     CUdeviceptr hflag_dev = 0;
+    CUstream arm = nullptr;   // CTXB_ARMED_SIGNAL: the library's signal stream
+    uint32_t gate_seq = 0;
   };
   std::vector<Res> pool;   // per-run device resources, reused (flag is always left at 0)
   uint32_t full_ir_words128() const {  // 128-B rows occupied by the FULL_IR layout
@@ -105,8 +107,11 @@ struct ctxb_run {
   uint64_t cbytes = 0, pay_off = 0, stride = 0;
   CUstream stream = nullptr;
   CUdeviceptr flag = 0, stamps = 0, forced = 0;
-  void* hflag = nullptr;    // CTXB_HOST_SIGNAL: preemption word in mapped pinned host memory
+  void* hflag = nullptr;    // mapped pinned host words: [0] CTXB_HOST_SIGNAL word, [16] CTXB_ARMED_SIGNAL gate
   CUdeviceptr hflag_dev = 0;
+  CUstream arm = nullptr;   // CTXB_ARMED_SIGNAL: stream holding the pre-enqueued signal
+  uint32_t gate_seq = 0;    //   gate value that releases the armed signal of the current launch
+  bool armed = false;       //   an armed signal is pending on `arm`
   uint32_t epoch = 0;
   uint32_t rb_target = 0;   // CTXB_GATHER_RESUME: blocks with preempted warps the resume launch waits for
   int state = RUN_RUNNING;
@@ -114,10 +119,22 @@ struct ctxb_run {
   bool resumed_launch = false;
   CUevent ev0 = nullptr, ev1 = nullptr;   // recorded around each launch on the run's stream
   CUevent evf = nullptr;                  // recorded on the control stream before the flag write
+  // CTXB_ARMED_SIGNAL: release a pending armed signal of a launch that was not
+  // preempted and clear the flag it raises (off the preemption path).
+  void disarm() {
+    if (!armed) return;
+    armed = false;
+    Driver& d = driver();
+    *(static_cast<volatile uint32_t*>(hflag) + 16) = gate_seq;
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    d.cuMemsetD32Async(flag, 0, 1, arm);
+    d.cuStreamSynchronize(arm);
+  }
   ~ctxb_run() {
     if (flag && prog) {   // return the resources to the program's pool
       std::lock_guard<std::mutex> g(prog->mu);
-      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf, hflag, hflag_dev});
+      disarm();
+      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf, hflag, hflag_dev, arm, gate_seq});
     }
   }
 };
@@ -284,6 +301,15 @@ int launch(ctxb_run* r, bool resume) {
   CU(d.cuLaunchKernel(resume ? r->mod.resume : r->mod.run, r->grid, 1, 1, (unsigned)r->prog->prog.block, 1, 1, 0,
                       r->stream, args, nullptr));
   CU(d.cuEventRecord(r->ev1, r->stream));
+  if (r->prog->opt.flags & CTXB_ARMED_SIGNAL) {
+    // pre-enqueue the signal behind a gate in mapped host memory: ctxb_preempt
+    // only stores the gate value, no driver call on the preemption path
+    r->gate_seq++;
+    CU(d.cuStreamWaitValue32(r->arm, r->hflag_dev + 64, r->gate_seq, CU_STREAM_WAIT_VALUE_GEQ));
+    CU(d.cuEventRecord(r->evf, r->arm));
+    CU(d.cuStreamWriteValue32(r->arm, r->flag, 1u, 0));
+    r->armed = true;
+  }
   r->state = RUN_RUNNING;
   r->resumed_launch = resume;
   return CTXB_OK;
@@ -292,6 +318,7 @@ int launch(ctxb_run* r, bool resume) {
 // Read the header array after the stream drained and classify the run.
 int collect(ctxb_run* r) {
   Driver& d = driver();
+  r->disarm();
   r->hdr_prev.swap(r->hdr);
   r->hdr.assign((size_t)r->n_warps * 4, 0);
   CU(d.cuMemcpyDtoHAsync(r->hdr.data(), r->cbuf, (size_t)r->n_warps * 16, r->stream));
@@ -329,7 +356,7 @@ int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb
   if (!ir_text || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   *out = nullptr;
   ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0};
-  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 1023 || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
+  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 2047 || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
     return fail(CTXB_E_INVALID_ARG, "bad options");
   std::unique_ptr<ctxb_program> p(new ctxb_program);
   p->opt = Options{o.flags, o.mode, o.poll_policy, o.poll_every ? o.poll_every : 8, o.debug,
@@ -373,6 +400,7 @@ int ctxb_program_destroy(ctxb_program* p) {
       d.cuEventDestroy(r.ev1);
       d.cuEventDestroy(r.evf);
       if (r.hflag) d.cuMemFreeHost(r.hflag);
+      if (r.arm) d.cuStreamDestroy(r.arm);
     }
   }
   delete p;
@@ -521,6 +549,8 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
         r->evf = p->pool[i].evf;
         r->hflag = p->pool[i].hflag;
         r->hflag_dev = p->pool[i].hflag_dev;
+        r->arm = p->pool[i].arm;
+        r->gate_seq = p->pool[i].gate_seq;
         p->pool.erase(p->pool.begin() + (long)i);
         break;
       }
@@ -540,12 +570,17 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
     std::vector<uint32_t> z(64 + grid, 0);
     CU(d.cuMemcpyHtoD(r->flag, z.data(), z.size() * 4));   // the flag is 0 whenever a run does not hold it raised
   }
-  if ((p->opt.flags & CTXB_HOST_SIGNAL) && !r->hflag) {
+  if ((p->opt.flags & (CTXB_HOST_SIGNAL | CTXB_ARMED_SIGNAL)) && !r->hflag) {
     void* h = nullptr;
     CU(d.cuMemHostAlloc(&h, 128, CU_MEMHOSTALLOC_DEVICEMAP | CU_MEMHOSTALLOC_PORTABLE));
     memset(h, 0, 128);
     r->hflag = h;
     CU(d.cuMemHostGetDevicePointer(&r->hflag_dev, h, 0));
+  }
+  if ((p->opt.flags & CTXB_ARMED_SIGNAL) && !r->arm) {
+    int lo = 0, hi = 0;
+    CU(d.cuCtxGetStreamPriorityRange(&lo, &hi));
+    CU(d.cuStreamCreateWithPriority(&r->arm, CU_STREAM_NON_BLOCKING, hi));
   }
   // No header memset: every warp of launch 0 writes its header (DONE or
   // PREEMPTED with epoch 1) before the launch completes.
@@ -564,7 +599,8 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
   if ((CUstream)ctrl == r->stream && ctrl != nullptr)
     return fail(CTXB_E_INVALID_ARG, "ctrl_stream must differ from the run's stream");
   Driver& d = driver();
-  volatile uint32_t* hf = static_cast<volatile uint32_t*>(r->hflag);
+  volatile uint32_t* hf =
+      (r->prog->opt.flags & CTXB_HOST_SIGNAL) ? static_cast<volatile uint32_t*>(r->hflag) : nullptr;
   double t0 = now_ms();
   if (hf) {
     // CTXB_HOST_SIGNAL: relay warps see this store over PCIe and raise the
@@ -576,13 +612,22 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
   // test knob: CTXB_HOST_SIGNAL_ONLY=1 drops the fallback, so the relay is the only path
   const char* ho = hf ? getenv("CTXB_HOST_SIGNAL_ONLY") : nullptr;
   const bool host_only = ho && atoi(ho) != 0;
-  CU(d.cuEventRecord(r->evf, (CUstream)ctrl));
-  if (!(hf && host_only)) CU(d.cuStreamWriteValue32((CUstream)ctrl, r->flag, 1u, 0));
+  CUstream cs = (CUstream)ctrl;
+  if (r->armed) {
+    // CTXB_ARMED_SIGNAL: release the signal enqueued on the library's stream at launch
+    *(static_cast<volatile uint32_t*>(r->hflag) + 16) = r->gate_seq;
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    r->armed = false;
+    cs = r->arm;
+  } else {
+    CU(d.cuEventRecord(r->evf, cs));
+    if (!(hf && host_only)) CU(d.cuStreamWriteValue32(cs, r->flag, 1u, 0));
+  }
   CU(d.cuStreamSynchronize(r->stream));
   double t1 = now_ms();
   if (hf) *hf = 0u;   // the victim has drained: no warp of this run reads it until the next launch
-  CU(d.cuMemsetD32Async(r->flag, 0, 1, (CUstream)ctrl));
-  CU(d.cuStreamSynchronize((CUstream)ctrl));
+  CU(d.cuMemsetD32Async(r->flag, 0, 1, cs));
+  CU(d.cuStreamSynchronize(cs));
   int rc = collect(r);
   if (rc) return rc;
   if (st) {
@@ -608,7 +653,6 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     }
     for (auto b : blk) st->blocks_preempted += b;
     st->latency_us = st->warps_preempted ? (double)(tmax - tmin) * 1e-3 : 0.0;
-    CU(d.cuStreamSynchronize((CUstream)ctrl));
     float ms = 0;
     CU(d.cuEventElapsedTime(&ms, r->evf, r->ev1));
     // with CTXB_HOST_SIGNAL the signal is the host store, which the event does not bound

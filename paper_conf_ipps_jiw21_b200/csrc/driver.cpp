@@ -54,9 +54,13 @@ Driver& driver() {
               sym(h, "cuStreamCreate", &d.cuStreamCreate, &e) && sym(h, "cuStreamDestroy_v2", &d.cuStreamDestroy, &e) &&
               sym(h, "cuMemcpyDtoHAsync_v2", &d.cuMemcpyDtoHAsync, &e) &&
               sym(h, "cuMemHostAlloc", &d.cuMemHostAlloc, &e) && sym(h, "cuMemFreeHost", &d.cuMemFreeHost, &e) &&
-              sym(h, "cuMemHostGetDevicePointer_v2", &d.cuMemHostGetDevicePointer, &e);
+              sym(h, "cuMemHostGetDevicePointer_v2", &d.cuMemHostGetDevicePointer, &e) &&
+              sym(h, "cuStreamCreateWithPriority", &d.cuStreamCreateWithPriority, &e) &&
+              sym(h, "cuCtxGetStreamPriorityRange", &d.cuCtxGetStreamPriorityRange, &e);
     if (ok && !sym(h, "cuStreamWriteValue32_v2", &d.cuStreamWriteValue32, &e))
       ok = sym(h, "cuStreamWriteValue32", &d.cuStreamWriteValue32, &e);
+    if (ok && !sym(h, "cuStreamWaitValue32_v2", &d.cuStreamWaitValue32, &e))
+      ok = sym(h, "cuStreamWaitValue32", &d.cuStreamWaitValue32, &e);
     if (!ok) return;
     CUresult r = d.cuInit(0);
     if (r != CUDA_SUCCESS) {

@@ -146,3 +146,16 @@ def test_host_signal_generates_and_compiles():
     f = cb.Program(txt, flags=cb.ALL | cb.HOST_SIGNAL, poll_policy=cb.POLL_EXPLICIT,
                    debug=cb.DEBUG_FORCED | cb.DEBUG_NO_COMPILE)
     assert "relay_fwd(hfl" not in f.source
+
+
+def test_armed_signal_is_runtime_only():
+    """CTXB_ARMED_SIGNAL is a runtime option: the generated
+    kernel source is byte-identical to the default build's."""
+    from workloads import configs
+    txt = configs.c3()["ir"]
+    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
+    armed = cb.Program(txt, flags=cb.ALL | cb.ARMED_SIGNAL, poll_policy=cb.POLL_EXPLICIT,
+                       debug=cb.DEBUG_NO_COMPILE)
+    assert armed.source == base.source
+    with pytest.raises(cb.CtxbError):
+        cb.Program(txt, flags=4096, debug=cb.DEBUG_NO_COMPILE)

@@ -213,7 +213,8 @@ def test_c2s_full_flag_equals_c2():
 
 
 @pytest.mark.parametrize("which,host", [("c2", False), ("c3", False), ("c2s", False),
-                                        ("c2", True), ("c3", True), ("c2s", True)])
+                                        ("c2", True), ("c3", True), ("c2s", True),
+                                        ("c2", "armed"), ("c3", "armed")])
 def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     """random flag times, repeated and nested
     preempt -> resume -> preempt ... cycles (each resume can be preempted
@@ -221,7 +222,9 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     the final output stays bit-exact with the uninterrupted run.  host=True:
     CTXB_HOST_SIGNAL with the stream-memop fallback disabled
     (CTXB_HOST_SIGNAL_ONLY=1), so every preemption arrives through a relay
-    warp's system-scope poll of the host word."""
+    warp's system-scope poll of the host word.  host="armed":
+    CTXB_ARMED_SIGNAL, every launch and resume pre-enqueues its signal behind
+    a host gate; runs that end unpreempted are disarmed."""
     import time
     import torch
     cb = _cb()
@@ -234,10 +237,10 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
         bufs = [to_dev(cfg["buffers"]["A"]), to_dev(cfg["buffers"]["B"]),
                 torch.zeros(4096 * 4096, dtype=torch.int32, device="cuda")]
         out_i, mb = 2, 2
-    if host:
+    if host is True:
         monkeypatch.setenv("CTXB_HOST_SIGNAL_ONLY", "1")
-    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=mb,
-                      flags=cb.ALL | (cb.HOST_SIGNAL if host else 0))
+    extra = cb.ARMED_SIGNAL if host == "armed" else cb.HOST_SIGNAL if host else 0
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=mb, flags=cb.ALL | extra)
     bps, nsm = prog.occupancy()
     grid = bps * nsm
     ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")

@@ -33,9 +33,11 @@ def setup(which):
     return cfg["ir"], lambda g: [a, b, torch.zeros(4096 * 4096, dtype=torch.int32, device="cuda")], 2, 0
 
 
-MODES = (("memop", 0, None, None), ("host R=1", cb.HOST_SIGNAL, "1", None),
-         ("host R=2", cb.HOST_SIGNAL, "2", None), ("host R=4", cb.HOST_SIGNAL, "4", None),
-         ("host R=1 only", cb.HOST_SIGNAL, "1", "1"))
+MODES = (("memop", 0, None, None), ("armed", cb.ARMED_SIGNAL, None, None),
+         ("host R=1", cb.HOST_SIGNAL, "1", None), ("armed + host R=1", cb.ARMED_SIGNAL | cb.HOST_SIGNAL, "1", None))
+if os.environ.get("ALL_MODES"):
+    MODES += (("host R=2", cb.HOST_SIGNAL, "2", None), ("host R=4", cb.HOST_SIGNAL, "4", None),
+              ("host R=1 only", cb.HOST_SIGNAL, "1", "1"))
 
 
 def main():
@@ -44,6 +46,7 @@ def main():
     rows = ["| config | signal | kernel ms (median of 5) | host latency µs p50 / p90 | signal->drained µs p50 (events) | "
             "routines µs p50 | flag-seen spread µs p50 | preempted |",
             "|---|---|---|---|---|---|---|---|"]
+    # host latency: ctxb_preempt entry -> victim drained (host clock); events: signal event -> drained
     for which in sys.argv[1:] or ["c2", "c3", "c4a"]:
         txt, mk, mb, extra = setup(which)
         for name, fl, relays, only in MODES:

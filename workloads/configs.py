@@ -84,7 +84,8 @@ def c2_ir(M=4096, N=4096, K=4096, unroll=4, polls="iter"):
     x`unroll` into one BB and software-pipelined: the fragments of step u+1 are
     loaded before the FFMAs of step u (the last prefetch of the final iteration
     is guarded off).  `poll` markers: polls="iter" -> one per iteration, after
-    the last FFMA (its window spans the whole unrolled iteration); "step" ->
+    the last FFMA (its window spans the whole unrolled iteration); "two" ->
+    before the FFMAs of steps 0 and unroll/2 (two sites per iteration); "step" ->
     before every step's FFMAs; "half" -> before and in the middle of every
     step's FFMAs.  Persistent grid: tile = ctaid + i*nctaid (reversible
     scalar IADD)."""
@@ -141,7 +142,7 @@ def c2_ir(M=4096, N=4096, K=4096, unroll=4, polls="iter"):
             loads(nxt, unroll, guard="s6")     # step 0 of the next iteration
         a, b = frag[cur]
         for q in range(64):
-            if polls in ("step", "half") and q == 0:
+            if (polls in ("step", "half") or (polls == "two" and u % (unroll // 2) == 0)) and q == 0:
                 e("  poll")
             if polls == "half" and q == 32:
                 e("  poll")
