@@ -54,6 +54,9 @@ def parse():
                     help="extra BASELINE configs measured after the C2 headline (comma list, or 'none')")
     ap.add_argument("--config-trials", type=int, default=5)
     ap.add_argument("--c5-seconds", type=float, default=4.0)
+    ap.add_argument("--signal", default="armed", choices=["armed", "memop"],
+                    help="C2 preemption signal of the headline modes: armed = CTXB_ARMED_SIGNAL (pre-enqueued "
+                         "behind a host gate, DESIGN.md 8j); memop = cuStreamWriteValue32 on the control stream")
     return ap.parse_args()
 
 
@@ -163,13 +166,17 @@ class Clocks:
 
 # ---- the GPU arm --------------------------------------------------------------
 
+SIGNAL_FLAGS = 0   # set by gpu_arm from --signal: cb.ARMED_SIGNAL or 0
+
+
 def make_c2(cb, size, mode, debug=0, flags=None):
     """C2 with one poll site per k-loop iteration (its window spans the whole
-    unrolled iteration) and 2 resident blocks / SM (__launch_bounds__)."""
+    unrolled iteration) and 2 resident blocks / SM (__launch_bounds__).
+    flags=None: CTXB_ALL plus the headline's signal option (--signal)."""
     from workloads import configs
     ir_text = configs.c2_ir(size, size, size, polls="iter")
     return cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, mode=mode, debug=debug, min_blocks_per_sm=2,
-                      flags=cb.ALL if flags is None else flags)
+                      flags=cb.ALL | SIGNAL_FLAGS if flags is None else flags)
 
 
 def spin_until(t):
@@ -250,6 +257,10 @@ def summarize(recs):
         out["header_bytes_per_tb"] = float(np.median([r["header"] / max(1, r["blocks"]) for r in pre]))
         out["insitu_save_gbs_median"] = float(np.median([r["payload"] / (r["latency_us"] * 1e3)
                                                          for r in pre if r["latency_us"] > 0]))
+        # every preempted warp reloads its payload between min t_resume_entry and max t_site_reached
+        rb = [r["payload"] / (r["resume_us"] * 1e3) for r in pre if r["resume_us"] > 0]
+        if rb:
+            out["insitu_restore_gbs_median"] = float(np.median(rb))
     return out
 
 
@@ -1000,6 +1011,8 @@ def gpu_arm(args):
     import torch
     import paper_conf_ipps_jiw21_b200 as cb
     from workloads import configs
+    global SIGNAL_FLAGS
+    SIGNAL_FLAGS = cb.ARMED_SIGNAL if args.signal == "armed" else 0
     ws, rank, local = dist_setup(args)
     torch.cuda.set_device(local)
     clk = Clocks(local)
@@ -1013,11 +1026,12 @@ def gpu_arm(args):
         progs["full_hw"] = make_c2(cb, size, cb.MODE_FULL_HW)
         progs["full_ir"] = make_c2(cb, size, cb.MODE_FULL)
         # CTXB_GATHER_RESUME: resumed warps wait until every preempted warp has restored
-        progs["ctxback_gather"] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | cb.GATHER_RESUME)
-        progs["full_hw_gather"] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | cb.GATHER_RESUME)
-        # CTXB_ARMED_SIGNAL: the signal is pre-enqueued at launch behind a host gate
-        progs["ctxback_armed"] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | cb.ARMED_SIGNAL)
-        progs["full_hw_armed"] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | cb.ARMED_SIGNAL)
+        progs["ctxback_gather"] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | cb.GATHER_RESUME | SIGNAL_FLAGS)
+        progs["full_hw_gather"] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | cb.GATHER_RESUME | SIGNAL_FLAGS)
+        # the other signal path next to the headline's
+        other, oname = (0, "memop") if SIGNAL_FLAGS else (cb.ARMED_SIGNAL, "armed")
+        progs["ctxback_" + oname] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | other)
+        progs["full_hw_" + oname] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | other)
     bps, nsm = progs["ctxback"].occupancy()
     for p in progs.values():
         bps = min(bps, p.occupancy()[0])
@@ -1052,7 +1066,8 @@ def gpu_arm(args):
     main = summarize(recs)
     # ---- baselines in the same framework (same fracs) ----
     base = {}
-    for k in ("full_hw", "full_ir", "live", "ctxback_gather", "full_hw_gather", "ctxback_armed", "full_hw_armed"):
+    for k in ("full_hw", "full_ir", "live", "ctxback_gather", "full_hw_gather", "ctxback_armed", "full_hw_armed",
+              "ctxback_memop", "full_hw_memop"):
         if k in progs:
             preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_w[:1], ws)
             r = preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_t, ws)
@@ -1148,9 +1163,10 @@ def gpu_arm(args):
                    "grid": grid, "block": 256, "t_uninterrupted_ms": round(t_unint_ms, 3),
                    "l2": "inputs larger than L2 (A, B, C = 192 MiB > 126 MB)", "parallelism": f"replicas x{ws}"},
         "resume_us": round(main["resume_us_median"], 3),
-        "value_definition": ("median over steps of signal -> all blocks drained: CUDA event on the control stream "
-                             "right before the flag write -> libctxb's event after the victim kernel (every warp "
-                             "saved or finished, kernel exited)"),
+        "value_definition": ("median over steps of signal -> all blocks drained: CUDA event right before the flag "
+                             "write on the signal's stream (--signal armed: libctxb's signal stream, the event runs "
+                             "once the host gate opened; memop: the caller's control stream) -> libctxb's event "
+                             "after the victim kernel (every warp saved or finished, kernel exited)"),
         "preemption_routines_us": round(main["latency_us_median"], 3),
         "preemption_routines_definition": "max t_saved - min t_flag_seen over preempted warps (%globaltimer)",
         "flag_propagation_us": {"median": round(prop_med, 3), "max": round(prop_max, 3),
@@ -1171,8 +1187,9 @@ def gpu_arm(args):
             "context_pct": (round(100 * (1 - main["context_bytes_per_tb"] / base["full_hw"]["context_bytes_per_tb"]), 2)
                             if "full_hw" in base and base["full_hw"].get("context_bytes_per_tb") and
                             main.get("context_bytes_per_tb") else None)},
-        "armed_reduction_vs_full_hw_armed": (_reduction(base, "ctxback_armed", "full_hw_armed")
-                                             if "ctxback_armed" in base and "full_hw_armed" in base else None),
+        "signal": args.signal,
+        "other_signal_reduction": {k: _reduction(base, "ctxback_" + k, "full_hw_" + k)
+                                   for k in ("armed", "memop") if "ctxback_" + k in base},
         "poll_overhead": ovh, "bulk": bulk, "configs": extra_cfg,
         "roofline": rf, "roofline_restore": rr,
         "cpu_baseline": cpu,
