@@ -283,9 +283,14 @@ int ctxb_launch(ctxb_program* prog, uint32_t grid_blocks, void* const* buffers,
                 const uint32_t* forced_targets, ctxb_run** out);
 
 /* Raise the preemption signal (a device flag written by `ctrl_stream`, which
- * must not be the run's stream), wait until every warp of the run has either
- * saved its context and exited or finished, clear the flag.  Fills
- * `stats` if non-NULL.  _STATE if the run is not running. */
+ * must not be the run's stream; with CTXB_ARMED_SIGNAL by the library's own
+ * stream), wait until every warp of the run has either saved its context and
+ * exited or finished, clear the flag.  Fills `stats` if non-NULL.
+ * stats == NULL returns as soon as the launch drained: the flag reset is
+ * ordered before the run's next launch on its stream, and the headers are
+ * read by the next call that needs the run's state (ctxb_wait / query /
+ * resume / read_*), so the GPU is free for other work one host round trip
+ * earlier.  _STATE if the run is not running. */
 int ctxb_preempt(ctxb_run* run, void* ctrl_stream, ctxb_preempt_stats* stats);
 
 /* Relaunch the same grid as a resume kernel: each preempted warp reloads its

@@ -67,6 +67,8 @@ struct ctxb_program {
     CUdeviceptr hflag_dev = 0;
     CUstream arm = nullptr;   // CTXB_ARMED_SIGNAL: the library's signal stream
     uint32_t gate_seq = 0;
+    CUevent evr = nullptr;    // flag reset recorded on the signal's stream
+    void* hdr_pin = nullptr;  // pinned staging for the header read-back
   };
   std::vector<Res> pool;   // per-run device resources, reused (flag is always left at 0)
   uint32_t full_ir_words128() const {  // 128-B rows occupied by the FULL_IR layout
@@ -94,7 +96,10 @@ struct ctxb_program {
   }
 };
 
-enum { RUN_RUNNING = 0, RUN_PREEMPTED = 1, RUN_DONE = 2 };
+// RUN_DRAINED: ctxb_preempt without stats returned as soon as the launch
+// drained; the headers are read (-> PREEMPTED / DONE) on the next call that
+// needs them (settle()).
+enum { RUN_RUNNING = 0, RUN_PREEMPTED = 1, RUN_DONE = 2, RUN_DRAINED = 3 };
 
 struct ctxb_run {
   ctxb_program* prog = nullptr;
@@ -119,6 +124,9 @@ struct ctxb_run {
   bool resumed_launch = false;
   CUevent ev0 = nullptr, ev1 = nullptr;   // recorded around each launch on the run's stream
   CUevent evf = nullptr;                  // recorded on the control stream before the flag write
+  CUevent evr = nullptr;                  // recorded after the flag reset on the signal's stream
+  bool reset_pending = false;             //   the next launch waits for it on its stream
+  void* hdr_pin = nullptr;                // pinned staging buffer for the headers (n_warps x 16 B)
   // CTXB_ARMED_SIGNAL: release a pending armed signal of a launch that was not
   // preempted and clear the flag it raises (off the preemption path).
   void disarm() {
@@ -134,7 +142,9 @@ struct ctxb_run {
     if (flag && prog) {   // return the resources to the program's pool
       std::lock_guard<std::mutex> g(prog->mu);
       disarm();
-      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf, hflag, hflag_dev, arm, gate_seq});
+      if (reset_pending) driver().cuEventSynchronize(evr);   // the flag is 0 again before it is reused
+      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf, hflag, hflag_dev, arm, gate_seq, evr,
+                            hdr_pin});
     }
   }
 };
@@ -297,6 +307,10 @@ int launch(ctxb_run* r, bool resume) {
   pack_params(r, r->prog, blob);
   void* args[] = {blob.data()};
   Driver& d = driver();
+  if (r->reset_pending) {   // the flag reset of the last preemption precedes this launch
+    CU(d.cuStreamWaitEvent(r->stream, r->evr, 0));
+    r->reset_pending = false;
+  }
   CU(d.cuEventRecord(r->ev0, r->stream));
   CU(d.cuLaunchKernel(resume ? r->mod.resume : r->mod.run, r->grid, 1, 1, (unsigned)r->prog->prog.block, 1, 1, 0,
                       r->stream, args, nullptr));
@@ -320,9 +334,10 @@ int collect(ctxb_run* r) {
   Driver& d = driver();
   r->disarm();
   r->hdr_prev.swap(r->hdr);
-  r->hdr.assign((size_t)r->n_warps * 4, 0);
-  CU(d.cuMemcpyDtoHAsync(r->hdr.data(), r->cbuf, (size_t)r->n_warps * 16, r->stream));
+  r->hdr.resize((size_t)r->n_warps * 4);
+  CU(d.cuMemcpyDtoHAsync(r->hdr_pin, r->cbuf, (size_t)r->n_warps * 16, r->stream));
   CU(d.cuStreamSynchronize(r->stream));
+  memcpy(r->hdr.data(), r->hdr_pin, (size_t)r->n_warps * 16);
   uint32_t pre = 0, done = 0;
   for (uint32_t w = 0; w < r->n_warps; w++) {
     const uint32_t* h = &r->hdr[(size_t)w * 4];
@@ -334,6 +349,12 @@ int collect(ctxb_run* r) {
                                  std::to_string(r->n_warps) + "): it faulted or was not launched");
   r->state = pre ? RUN_PREEMPTED : RUN_DONE;
   return CTXB_OK;
+}
+
+// Classify a launch that ctxb_preempt left drained but not collected.
+int settle(const ctxb_run* cr) {
+  ctxb_run* r = const_cast<ctxb_run*>(cr);
+  return r->state == RUN_DRAINED ? collect(r) : CTXB_OK;
 }
 
 template <class T>
@@ -401,6 +422,8 @@ int ctxb_program_destroy(ctxb_program* p) {
       d.cuEventDestroy(r.evf);
       if (r.hflag) d.cuMemFreeHost(r.hflag);
       if (r.arm) d.cuStreamDestroy(r.arm);
+      d.cuEventDestroy(r.evr);
+      if (r.hdr_pin) d.cuMemFreeHost(r.hdr_pin);
     }
   }
   delete p;
@@ -551,6 +574,8 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
         r->hflag_dev = p->pool[i].hflag_dev;
         r->arm = p->pool[i].arm;
         r->gate_seq = p->pool[i].gate_seq;
+        r->evr = p->pool[i].evr;
+        r->hdr_pin = p->pool[i].hdr_pin;
         p->pool.erase(p->pool.begin() + (long)i);
         break;
       }
@@ -567,6 +592,8 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
     CU(d.cuEventCreate(&r->ev0, CU_EVENT_DEFAULT));
     CU(d.cuEventCreate(&r->ev1, CU_EVENT_DEFAULT));
     CU(d.cuEventCreate(&r->evf, CU_EVENT_DEFAULT));
+    CU(d.cuEventCreate(&r->evr, CU_EVENT_DISABLE_TIMING));
+    CU(d.cuMemHostAlloc(&r->hdr_pin, (size_t)r->n_warps * 16, 0));
     std::vector<uint32_t> z(64 + grid, 0);
     CU(d.cuMemcpyHtoD(r->flag, z.data(), z.size() * 4));   // the flag is 0 whenever a run does not hold it raised
   }
@@ -627,10 +654,18 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
   double t1 = now_ms();
   if (hf) *hf = 0u;   // the victim has drained: no warp of this run reads it until the next launch
   CU(d.cuMemsetD32Async(r->flag, 0, 1, cs));
+  if (!st) {
+    // return at once: the next launch waits for the reset on its own stream,
+    // and the headers are read when first needed (settle)
+    CU(d.cuEventRecord(r->evr, cs));
+    r->reset_pending = true;
+    r->state = RUN_DRAINED;
+    return CTXB_OK;
+  }
   CU(d.cuStreamSynchronize(cs));
   int rc = collect(r);
   if (rc) return rc;
-  if (st) {
+  {
     memset(st, 0, sizeof *st);
     st->host_us = (t1 - t0) * 1e3;
     std::vector<uint64_t> stamps((size_t)r->n_warps * 4);
@@ -663,6 +698,7 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
 
 int ctxb_resume(ctxb_run* r, void* stream, const uint32_t* forced_targets) {
   if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
+  if (int rc = settle(r)) return rc;
   if (r->state != RUN_PREEMPTED) return fail(CTXB_E_STATE, "run is not preempted");
   r->stream = (CUstream)stream;
   int rc = upload_forced(r, forced_targets);
@@ -695,6 +731,7 @@ int ctxb_resume(ctxb_run* r, void* stream, const uint32_t* forced_targets) {
 
 int ctxb_wait(ctxb_run* r, int* finished) {
   if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
+  if (int rc = settle(r)) return rc;
   if (r->state == RUN_RUNNING) {
     CU(driver().cuStreamSynchronize(r->stream));
     int rc = collect(r);
@@ -706,6 +743,7 @@ int ctxb_wait(ctxb_run* r, int* finished) {
 
 int ctxb_query(ctxb_run* r, int* running) {
   if (!r || !running) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  if (int rc = settle(r)) return rc;
   if (r->state != RUN_RUNNING) {
     *running = 0;
     return CTXB_OK;
@@ -827,6 +865,7 @@ int ctxb_flag_propagation(void* ctrl, uint32_t trials, double* median_us, double
 
 int ctxb_launch_ms(const ctxb_run* r, float* ms) {
   if (!r || !ms) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  if (int rc = settle(r)) return rc;
   if (r->state == RUN_RUNNING) return fail(CTXB_E_STATE, "launch still running: call ctxb_wait/ctxb_preempt first");
   Driver& d = driver();
   CU(d.cuEventSynchronize(r->ev1));
@@ -836,6 +875,7 @@ int ctxb_launch_ms(const ctxb_run* r, float* ms) {
 
 int ctxb_resume_stats_get(const ctxb_run* r, ctxb_resume_stats* o) {
   if (!r || !o) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  if (int rc = settle(r)) return rc;
   memset(o, 0, sizeof *o);
   if (!r->resumed_launch || r->state == RUN_RUNNING || r->hdr_prev.empty()) return CTXB_OK;
   std::vector<uint64_t> stamps((size_t)r->n_warps * 4);
@@ -855,6 +895,7 @@ int ctxb_resume_stats_get(const ctxb_run* r, ctxb_resume_stats* o) {
 
 int ctxb_context_bytes(const ctxb_run* r, uint64_t* payload, uint64_t* header, uint32_t* n_tb) {
   if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
+  if (int rc = settle(r)) return rc;
   uint64_t pb = 0, hb = 0;
   uint32_t nwb = r->prog->prog.block / 32;
   std::vector<uint8_t> blk(r->grid, 0);
@@ -876,6 +917,7 @@ int ctxb_context_bytes(const ctxb_run* r, uint64_t* payload, uint64_t* header, u
 
 int ctxb_read_headers(const ctxb_run* r, uint32_t* out, uint64_t n) {
   if (!r || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  if (int rc = settle(r)) return rc;
   if (n < (uint64_t)r->n_warps * 4) return fail(CTXB_E_BUFFER_TOO_SMALL, "need 4 words per warp");
   if (r->hdr.empty()) return fail(CTXB_E_STATE, "no completed launch yet");
   memcpy(out, r->hdr.data(), (size_t)r->n_warps * 16);
@@ -884,6 +926,7 @@ int ctxb_read_headers(const ctxb_run* r, uint32_t* out, uint64_t n) {
 
 int ctxb_read_stamps(const ctxb_run* r, uint64_t* out, uint64_t n) {
   if (!r || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  if (int rc = settle(r)) return rc;
   if (n < (uint64_t)r->n_warps * 4) return fail(CTXB_E_BUFFER_TOO_SMALL, "need 4 words per warp");
   CU(driver().cuMemcpyDtoH(out, r->stamps, (size_t)r->n_warps * 32));
   return CTXB_OK;

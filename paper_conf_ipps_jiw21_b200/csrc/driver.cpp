@@ -56,7 +56,8 @@ Driver& driver() {
               sym(h, "cuMemHostAlloc", &d.cuMemHostAlloc, &e) && sym(h, "cuMemFreeHost", &d.cuMemFreeHost, &e) &&
               sym(h, "cuMemHostGetDevicePointer_v2", &d.cuMemHostGetDevicePointer, &e) &&
               sym(h, "cuStreamCreateWithPriority", &d.cuStreamCreateWithPriority, &e) &&
-              sym(h, "cuCtxGetStreamPriorityRange", &d.cuCtxGetStreamPriorityRange, &e);
+              sym(h, "cuCtxGetStreamPriorityRange", &d.cuCtxGetStreamPriorityRange, &e) &&
+              sym(h, "cuStreamWaitEvent", &d.cuStreamWaitEvent, &e);
     if (ok && !sym(h, "cuStreamWriteValue32_v2", &d.cuStreamWriteValue32, &e))
       ok = sym(h, "cuStreamWriteValue32", &d.cuStreamWriteValue32, &e);
     if (ok && !sym(h, "cuStreamWaitValue32_v2", &d.cuStreamWaitValue32, &e))

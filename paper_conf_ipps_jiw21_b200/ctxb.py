@@ -293,10 +293,30 @@ class Run:
     def n_warps(self):
         return self.grid * self.prog.info["block"] // 32
 
-    def preempt(self, ctrl_stream):
+    def preempt(self, ctrl_stream, stats=True):
+        """Raise the signal and wait until the launch drained (ctxb_preempt).
+        stats=False passes NULL stats (no stamp read-back on the preemption
+        path) and returns None: `finished` tells whether warps were
+        preempted, drain_stats() computes the device numbers later."""
+        if not stats:
+            _chk(lib.ctxb_preempt(self._h, _stream(ctrl_stream), None))
+            return None
         s = _PreStats()
         _chk(lib.ctxb_preempt(self._h, _stream(ctrl_stream), C.byref(s)))
         return {k: getattr(s, k) for k, _ in _PreStats._fields_}
+
+    def drain_stats(self):
+        """Device numbers of the last preempted launch, from the headers and
+        %globaltimer stamps (as ctxb_preempt computes them): warps / blocks
+        preempted, payload bytes, routines span max t_saved - min t_flag_seen."""
+        h = self.headers()
+        pre = h[:, 2] == STATE_PREEMPTED      # a PREEMPTED header always belongs to the latest launch
+        out = {"warps_preempted": int(pre.sum()), "payload_bytes": int(h[pre, 1].astype(np.uint64).sum()),
+               "blocks_preempted": int(pre.reshape(self.grid, -1).any(axis=1).sum()), "latency_us": 0.0}
+        if out["warps_preempted"]:
+            st = self.stamps()[pre].astype(np.int64)
+            out["latency_us"] = float(st[:, 1].max() - st[:, 0].min()) / 1e3
+        return out
 
     def resume(self, stream=None, forced=None):
         f = _u32arr(forced)

@@ -275,3 +275,48 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
         torch.cuda.synchronize()
         assert torch.equal(bufs[out_i], ref), f"{which}: output differs after {cycles} nested cycles"
     assert cycles >= 3 and total_pre > 0
+
+
+@pytest.mark.parametrize("armed", [False, True])
+def test_statless_preempt_settles_lazily(armed):
+    """ctxb_preempt with NULL stats returns once drained (state settled on the
+    next call): repeated nested cycles on C3 with stats=False stay bit-exact,
+    drain_stats() matches the header counts, and a finished run reports done."""
+    import time
+    import torch
+    cb = _cb()
+    cfg = configs.c3()
+    bufs = [to_dev(cfg["buffers"]["X"]), torch.zeros(cfg["W"] * cfg["H"], dtype=torch.int32, device="cuda")]
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | (cb.ARMED_SIGNAL if armed else 0))
+    bps, nsm = prog.occupancy()
+    grid = bps * nsm
+    ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
+    run = prog.launch(grid, bufs, [], ctx, s)
+    assert run.wait()
+    T = run.launch_ms() / 1e3
+    ref = bufs[1].clone()
+    rng = np.random.default_rng(5)
+    npre = 0
+    for trial in range(4):
+        bufs[1].zero_()
+        torch.cuda.synchronize()
+        run = prog.launch(grid, bufs, [], ctx, s)
+        for _ in range(6):
+            t0 = time.perf_counter()
+            while time.perf_counter() < t0 + rng.uniform(0.05, 0.3) * T:
+                pass
+            assert run.preempt(ctrl, stats=False) is None
+            if run.finished:
+                break
+            d = run.drain_stats()
+            h = run.headers()
+            assert d["warps_preempted"] == int((h[:, 2] == 1).sum()) > 0
+            assert d["payload_bytes"] == int(h[h[:, 2] == 1, 1].astype(np.int64).sum())
+            npre += d["warps_preempted"]
+            run.resume(s)
+        while not run.wait():
+            run.resume(s)
+        torch.cuda.synchronize()
+        assert torch.equal(bufs[1], ref)
+    assert npre > 0
