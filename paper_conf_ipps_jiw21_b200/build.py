@@ -29,7 +29,7 @@ def build(force=False, verbose=True):
     if not force and not needs_build():
         return OUT
     cmd = ["g++", "-O2", "-g", "-std=c++17", "-fPIC", "-shared", "-Wall", "-Wno-format-truncation",
-           f"-I{CUDA}/include", "-o", OUT + ".tmp"] + [os.path.join(CSRC, s) for s in SOURCES] + ["-ldl"]
+           f"-I{CUDA}/include", "-o", OUT + ".tmp"] + [os.path.join(CSRC, s) for s in SOURCES] + ["-ldl", "-pthread"]
     if verbose:
         print(" ".join(cmd), file=sys.stderr)
     subprocess.check_call(cmd)

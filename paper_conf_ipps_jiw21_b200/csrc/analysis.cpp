@@ -10,9 +10,13 @@
 //   least-latency flashback-point per instruction ................... P:313, P:337 (R-10)
 //   context incl. results restored by saving/reloading .............. P:343 (R-8)
 #include <algorithm>
+#include <atomic>
+#include <cstdlib>
+#include <exception>
 #include <functional>
 #include <set>
 #include <sstream>
+#include <thread>
 
 #include "ctxb_internal.h"
 
@@ -1076,6 +1080,40 @@ static std::vector<int> defer_targets(const Program& P, const Analysis& A, uint3
 
 static Analysis analyze_plans(const Program& P, const Options& opt);
 
+// Sites are independent given the backups (each evaluates its own windows),
+// so the per-site searches run on host threads; every result lands in its
+// own slot, so the analysis is identical for any thread count.  Threads:
+// env CTXB_ANALYZE_THREADS, default min(hardware threads, 16); 1 = serial.
+static unsigned analyze_threads() {
+  const char* e = getenv("CTXB_ANALYZE_THREADS");
+  unsigned v = e ? (unsigned)strtoul(e, nullptr, 10) : std::min(16u, std::thread::hardware_concurrency());
+  return std::max(1u, std::min(v, 256u));
+}
+
+static void parallel_for(size_t n, unsigned nt, const std::function<void(size_t, unsigned)>& fn) {
+  unsigned t = (unsigned)std::min<size_t>(nt, n);
+  if (t <= 1) {
+    for (size_t i = 0; i < n; i++) fn(i, 0);
+    return;
+  }
+  std::atomic<size_t> next{0};
+  std::vector<std::exception_ptr> err(t);
+  std::vector<std::thread> th;
+  for (unsigned w = 0; w < t; w++)
+    th.emplace_back([&, w] {
+      try {
+        // last index first: later sites of a basic block have more windows
+        for (size_t i; (i = next.fetch_add(1)) < n;) fn(n - 1 - i, w);
+      } catch (...) {
+        err[w] = std::current_exception();
+        next = n;
+      }
+    });
+  for (auto& x : th) x.join();
+  for (auto& e : err)
+    if (e) std::rethrow_exception(e);
+}
+
 Analysis analyze(const Program& P, const Options& opt) {
   Analysis A = analyze_plans(P, opt);
   if (opt.flags & F_DEFER) {
@@ -1111,32 +1149,45 @@ static Analysis analyze_plans(const Program& P, const Options& opt0) {
     return A;
   }
   uint32_t fl = opt.flags;
+  const unsigned nt = analyze_threads();
   if ((fl & F_OSRB) && (fl & F_RELAXED)) {
     // R-7 selects backups by the bytes of the greedy R-10 choice, whatever the
     // ranking or the plan search (R-19)
     uint32_t fb = fl & ~(F_RANK_RESUME | F_EXACT);
-    std::map<int, uint32_t> base;
-    for (int c : A.sites) base[c] = best_plan(P, L, D, A.heads, c, {}, fb).payload_bytes;
+    std::vector<uint32_t> base(A.sites.size());
+    parallel_for(A.sites.size(), nt, [&](size_t k, unsigned) {
+      base[k] = best_plan(P, L, D, A.heads, A.sites[k], {}, fb).payload_bytes;
+    });
     for (int m : osrb_candidates(P)) {
+      // m is selected if it shrinks the plan of any site after it in its window
       int bbm = P.bb_of[m];
-      for (int c : A.sites) {
-        if (c >= (int)P.ins.size() || P.bb_of[c] != bbm || c <= m || A.heads[c] > m) continue;
-        if (best_plan(P, L, D, A.heads, c, {m}, fb).payload_bytes < base[c]) {
-          A.backups.push_back(m);
-          break;
-        }
+      std::vector<size_t> ks;
+      for (size_t k = 0; k < A.sites.size(); k++) {
+        int c = A.sites[k];
+        if (c < (int)P.ins.size() && P.bb_of[c] == bbm && c > m && A.heads[c] <= m) ks.push_back(k);
       }
+      std::atomic<bool> gain{false};
+      parallel_for(ks.size(), nt, [&](size_t i, unsigned) {
+        if (gain.load()) return;
+        if (best_plan(P, L, D, A.heads, A.sites[ks[i]], {m}, fb).payload_bytes < base[ks[i]]) gain = true;
+      });
+      if (gain) A.backups.push_back(m);
     }
   }
-  ExactCfg ex;
-  if (opt.exact_budget) ex.budget = opt.exact_budget;
-  for (int c : A.sites)
-    A.plans.push_back(
-        best_plan(P, L, D, A.heads, c, A.backups, fl, opt.defer_instr_bytes, opt.resume_level_bytes, &ex));
-  A.exact_windows = ex.windows;
-  A.exact_truncated = ex.truncated;
-  A.exact_improved = ex.improved;
-  A.exact_fallback = ex.fallback;
+  std::vector<ExactCfg> ex(nt);
+  for (auto& e : ex)
+    if (opt.exact_budget) e.budget = opt.exact_budget;
+  A.plans.resize(A.sites.size());
+  parallel_for(A.sites.size(), nt, [&](size_t k, unsigned w) {
+    A.plans[k] = best_plan(P, L, D, A.heads, A.sites[k], A.backups, fl, opt.defer_instr_bytes,
+                           opt.resume_level_bytes, &ex[w]);
+  });
+  for (auto& e : ex) {
+    A.exact_windows += e.windows;
+    A.exact_truncated += e.truncated;
+    A.exact_improved += e.improved;
+    A.exact_fallback += e.fallback;
+  }
   return A;
 }
 

@@ -187,6 +187,61 @@ int ensure_module(ctxb_program* p, CUcontext c, Mod* out) {
   return CTXB_OK;
 }
 
+// Register count of kernel `fn` from the cubin itself: the EIATTR_REGCOUNT
+// attribute (0x2f, EIFMT_SVAL payload {u32 symbol index, u32 count}) of the
+// ELF's ".nv.info" section, the symbol named through .symtab/.strtab.  (The
+// ptxas -v text in the NVRTC log is not always there: it is missing when the
+// process runs under ncu.)  Returns 0 if absent or malformed.
+uint32_t cubin_regcount(const std::vector<char>& cb, const char* fn) {
+  auto rd = [&](size_t o, size_t n, void* out) {
+    if (o + n > cb.size()) return false;
+    memcpy(out, cb.data() + o, n);
+    return true;
+  };
+  uint64_t shoff = 0;
+  uint16_t shent = 0, shnum = 0, shstr = 0;
+  if (cb.size() < 64 || memcmp(cb.data(), "\x7f" "ELF", 4) != 0 || !rd(0x28, 8, &shoff) || !rd(0x3A, 2, &shent) ||
+      !rd(0x3C, 2, &shnum) || !rd(0x3E, 2, &shstr) || shent < 64 || shstr >= shnum)
+    return 0;
+  struct Sec { uint32_t name = 0; uint64_t off = 0, size = 0; uint32_t link = 0; };
+  std::vector<Sec> s(shnum);
+  for (uint32_t i = 0; i < shnum; i++) {
+    size_t o = shoff + (size_t)i * shent;
+    if (!rd(o, 4, &s[i].name) || !rd(o + 0x18, 8, &s[i].off) || !rd(o + 0x20, 8, &s[i].size) ||
+        !rd(o + 0x28, 4, &s[i].link))
+      return 0;
+  }
+  auto str = [&](uint64_t base, uint32_t o) -> std::string {
+    std::string out;
+    for (size_t i = base + o; i < cb.size() && cb[i]; i++) out += cb[i];
+    return out;
+  };
+  int info = -1, sym = -1;
+  for (uint32_t i = 0; i < shnum; i++) {
+    std::string nm = str(s[shstr].off, s[i].name);
+    if (nm == ".nv.info") info = (int)i;
+    if (nm == ".symtab") sym = (int)i;
+  }
+  if (info < 0 || sym < 0 || s[sym].link >= shnum) return 0;
+  const Sec& st = s[s[sym].link];
+  for (uint64_t i = s[info].off, end = s[info].off + s[info].size; i + 4 <= end;) {
+    uint8_t fmt = (uint8_t)cb[i], attr = (uint8_t)cb[i + 1];
+    uint16_t sz = 0;
+    if (fmt != 0x04) {   // NVAL / BVAL / HVAL: 4 bytes
+      i += 4;
+      continue;
+    }
+    if (!rd(i + 2, 2, &sz)) return 0;
+    if (attr == 0x2f && sz >= 8) {
+      uint32_t si = 0, cnt = 0, nmo = 0;
+      if (!rd(i + 4, 4, &si) || !rd(i + 8, 4, &cnt) || !rd(s[sym].off + (uint64_t)si * 24, 4, &nmo)) return 0;
+      if (str(st.off, nmo) == fn) return cnt;
+    }
+    i += 4 + sz;
+  }
+  return 0;
+}
+
 int nvrtc_compile(ctxb_program* p, uint32_t* regs_run, uint32_t* regs_resume) {
   Nvrtc& n = nvrtc();
   if (!n.ok) return fail(CTXB_E_NVRTC, n.err);
@@ -219,8 +274,16 @@ int nvrtc_compile(ctxb_program* p, uint32_t* regs_run, uint32_t* regs_resume) {
     if (std::regex_search(tail, m, std::regex("Used ([0-9]+) registers"))) return (uint32_t)std::stoul(m[1]);
     return 0;
   };
-  *regs_run = regs_of("ctxb_run");
-  *regs_resume = regs_of("ctxb_resume");
+  *regs_run = cubin_regcount(p->cubin, "ctxb_run");
+  *regs_resume = cubin_regcount(p->cubin, "ctxb_resume");
+  // the two sources must agree when the log has them
+  uint32_t lr = regs_of("ctxb_run"), ls2 = regs_of("ctxb_resume");
+  if ((lr && lr != *regs_run) || (ls2 && ls2 != *regs_resume))
+    return fail(CTXB_E_NVRTC, "register counts: cubin " + std::to_string(*regs_run) + "/" +
+                                  std::to_string(*regs_resume) + " vs ptxas log " + std::to_string(lr) + "/" +
+                                  std::to_string(ls2));
+  if (!*regs_run) *regs_run = lr;
+  if (!*regs_resume) *regs_resume = ls2;
   return CTXB_OK;
 }
 

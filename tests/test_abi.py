@@ -159,3 +159,20 @@ def test_armed_signal_is_runtime_only():
     assert armed.source == base.source
     with pytest.raises(cb.CtxbError):
         cb.Program(txt, flags=4096, debug=cb.DEBUG_NO_COMPILE)
+
+
+@pytest.mark.parametrize("flags", [cb.ALL, cb.ALL | cb.EXACT, cb.ALL | cb.RANK_RESUME | cb.PRUNE])
+def test_parallel_analysis_equals_serial(flags, monkeypatch):
+    """The per-site searches run on host threads (CTXB_ANALYZE_THREADS); plans,
+    OSRB backups and exact-search counters equal the serial analysis."""
+    txts = [configs.c4a_ir(1 << 14), configs.c3(512, 128, 64)["ir"]] + \
+        [random_program(900 + s, loop=True, n_body=16)[0] for s in range(3)]
+    for txt in txts:
+        out = []
+        for nt in ("1", "7"):
+            monkeypatch.setenv("CTXB_ANALYZE_THREADS", nt)
+            p = cb.Program(txt, flags=flags, debug=cb.DEBUG_NO_COMPILE)
+            i = p.info
+            out.append(([p.plan_text(k) for k in range(p.num_sites)], p.backups,
+                        [i[k] for k in ("exact_windows", "exact_truncated", "exact_improved", "exact_fallback")]))
+        assert out[0] == out[1]
