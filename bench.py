@@ -54,6 +54,9 @@ def parse():
                     help="extra BASELINE configs measured after the C2 headline (comma list, or 'none')")
     ap.add_argument("--config-trials", type=int, default=5)
     ap.add_argument("--c5-seconds", type=float, default=4.0)
+    ap.add_argument("--warm-resume", action="store_true",
+                    help="do not evict L2 between preempt and resume (default: 256 MiB written on the run's "
+                         "stream, standing in for the LS job, so the context is read back from HBM)")
     ap.add_argument("--signal", default="armed", choices=["armed", "memop"],
                     help="C2 preemption signal of the headline modes: armed = CTXB_ARMED_SIGNAL (pre-enqueued "
                          "behind a host gate, DESIGN.md 8j); memop = cuStreamWriteValue32 on the control stream")
@@ -179,6 +182,23 @@ def make_c2(cb, size, mode, debug=0, flags=None):
                       flags=cb.ALL | SIGNAL_FLAGS if flags is None else flags)
 
 
+_L2_SCRATCH = []
+WARM_RESUME = False   # --warm-resume: skip the eviction (context still L2-resident at resume)
+
+
+def evict_l2(stream):
+    """Between preempt and resume: write 256 MiB (> the 126 MB L2) on the
+    run's stream, standing in for the latency-sensitive job that runs there in
+    a real preemption, so the resume reads its context from HBM."""
+    import torch
+    if WARM_RESUME:
+        return
+    if not _L2_SCRATCH:
+        _L2_SCRATCH.append(torch.empty(64 << 20, dtype=torch.int32, device="cuda"))
+    with torch.cuda.stream(stream):
+        _L2_SCRATCH[0].fill_(len(_L2_SCRATCH))
+
+
 def spin_until(t):
     while time.perf_counter() < t:
         pass
@@ -208,6 +228,7 @@ def preempt_steps(cb, prog, grid, bufs, ctx, s, ctrl, ref, t_unint_s, fracs, ws,
         if st["warps_preempted"]:
             hdr = run.headers().copy()
             pre = (hdr[:, 2] == 1) & (hdr[:, 3] == 1)
+            evict_l2(s)
             run.resume(s)
             run.wait()
             launches += 1
@@ -467,6 +488,7 @@ def _flag_trials(progs, grid, make_bufs, uniforms, check, fracs, T_s):
             if st["warps_preempted"]:
                 hdr = run.headers().copy()
                 pre = (hdr[:, 2] == 1) & (hdr[:, 3] == 1)
+                evict_l2(s)
                 run.resume(s)
                 run.wait()
                 rs = run.resume_stats()
@@ -696,6 +718,7 @@ def bench_c4b(cb, trials, seed):
                     st = run.preempt(ctrl)
                     rs = {"resume_us": 0.0}
                     if st["warps_preempted"]:
+                        evict_l2(s)
                         run.resume(s)
                         run.wait()
                         rs = run.resume_stats()
@@ -1047,8 +1070,9 @@ def gpu_arm(args):
     import torch
     import paper_conf_ipps_jiw21_b200 as cb
     from workloads import configs
-    global SIGNAL_FLAGS
+    global SIGNAL_FLAGS, WARM_RESUME
     SIGNAL_FLAGS = cb.ARMED_SIGNAL if args.signal == "armed" else 0
+    WARM_RESUME = args.warm_resume
     ws, rank, local = dist_setup(args)
     torch.cuda.set_device(local)
     clk = Clocks(local)
@@ -1197,7 +1221,11 @@ def gpu_arm(args):
         "config": {"workload": f"C2 tiled SGEMM IR kernel {M}x{N}x{K} f32 (configs[1]), persistent grid "
                                f"{nsm} SMs x {bps} blocks x 256 threads, flag at U[0.05,0.95] x T_uninterrupted",
                    "grid": grid, "block": 256, "t_uninterrupted_ms": round(t_unint_ms, 3),
-                   "l2": "inputs larger than L2 (A, B, C = 192 MiB > 126 MB)", "parallelism": f"replicas x{ws}"},
+                   "l2": "inputs larger than L2 (A, B, C = 192 MiB > 126 MB)",
+                   "resume_l2": ("warm: context still L2-resident at resume" if args.warm_resume else
+                                 "cold: 256 MiB written on the run's stream between preempt and resume (stands in "
+                                 "for the LS job), so every resume reads its context from HBM"),
+                   "parallelism": f"replicas x{ws}"},
         "resume_us": round(main["resume_us_median"], 3),
         "value_definition": ("median over steps of signal -> all blocks drained: CUDA event right before the flag "
                              "write on the signal's stream (--signal armed: libctxb's signal stream, the event runs "
