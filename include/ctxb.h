@@ -127,6 +127,12 @@ extern "C" {
                              ctxb_query / destroy).  Kernels are unchanged.
                              signal_to_drained_us = signal event (after the
                              gate opened) -> victim drained    */
+#define CTXB_OSRB_SMEM  2048u /* codegen: OSRB backups live in a
+                             per-warp shared-memory slot (the paper's LDS
+                             tier: 4 B per backup per warp) instead of a
+                             register (4 B per backup per thread); every lane
+                             stores the warp-uniform value, each reads its own
+                             write.  Plans and bytes unchanged               */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */

@@ -176,3 +176,16 @@ def test_parallel_analysis_equals_serial(flags, monkeypatch):
             out.append(([p.plan_text(k) for k in range(p.num_sites)], p.backups,
                         [i[k] for k in ("exact_windows", "exact_truncated", "exact_improved", "exact_fallback")]))
         assert out[0] == out[1]
+
+
+def test_osrb_smem_slots_generate_and_compile():
+    """CTXB_OSRB_SMEM moves the OSRB backup of C4a into a per-warp shared
+    slot: plans unchanged, no bk register left, compiles for sm_100a."""
+    txt = configs.c4a_ir(1 << 14)
+    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
+    s = cb.Program(txt, flags=cb.ALL | cb.OSRB_SMEM, poll_policy=cb.POLL_EXPLICIT)
+    assert s.info["compiled"] == 1 and s.backups == base.backups and s.backups
+    assert [s.plan_text(k) for k in range(s.num_sites)] == [base.plan_text(k) for k in range(base.num_sites)]
+    m = s.backups[0]
+    assert f"BKS[warp][0] = " in s.source and f"u32 bk{m} " not in s.source
+    assert f"u32 bk{m} = 0u;" in base.source

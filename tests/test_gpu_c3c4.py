@@ -24,11 +24,11 @@ def _cb():
     return cb
 
 
-def forced_parity(cfg, grid, nsched, max_visit, skip=(), compare=None, seed=5, flags=7):
+def forced_parity(cfg, grid, nsched, max_visit, skip=(), compare=None, seed=5, flags=7, prog_flags=0):
     cb = _cb()
     op = ir.parse(cfg["ir"])
     an = A.analyze(op, policy="EXPLICIT", flags=flags)
-    prog = cb.Program(cfg["ir"], flags=flags, poll_policy=cb.POLL_EXPLICIT,
+    prog = cb.Program(cfg["ir"], flags=flags | prog_flags, poll_policy=cb.POLL_EXPLICIT,
                       debug=cb.DEBUG_FORCED | cb.DEBUG_POISON)
     for k, c in enumerate(an.sites):
         assert prog.plan_text(k) == A.plan_text(op, an.plans[c])
@@ -69,9 +69,10 @@ def test_c3_small_forced_rank_resume():
     assert all(an.plans[c].p == c for c in an.sites)
 
 
-def test_c4a_small_forced():
+@pytest.mark.parametrize("smem", [False, True])
+def test_c4a_small_forced(smem):
     cfg = configs.c4a(1 << 14, grid=2)
-    an = forced_parity(cfg, 2, 3, 4)
+    an = forced_parity(cfg, 2, 3, 4, prog_flags=2048 if smem else 0)   # 2048 = CTXB_OSRB_SMEM
     assert an.backups, "C4a must select an OSRB backup"
 
 

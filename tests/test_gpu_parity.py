@@ -28,13 +28,14 @@ def _cb():
 
 
 def check(txt, grid, bufs, schedules, policy="EVERY_INSTR", skip=("scr",), poison=True, flags=7, mode=0,
-          defer_instr_bytes=8):
+          defer_instr_bytes=8, runtime_flags=0):
     cb = _cb()
     op = ir.parse(txt)
     an = A.analyze(op, policy=policy, flags=flags, mode=mode, defer_instr_bytes=defer_instr_bytes)
     pol = {"EVERY_INSTR": cb.POLL_EVERY_INSTR, "EXPLICIT": cb.POLL_EXPLICIT}[policy]
     dbg = cb.DEBUG_FORCED | (cb.DEBUG_POISON if poison else 0)
-    prog = cb.Program(txt, flags=flags, poll_policy=pol, debug=dbg, mode=mode, defer_instr_bytes=defer_instr_bytes)
+    prog = cb.Program(txt, flags=flags | runtime_flags, poll_policy=pol, debug=dbg, mode=mode,
+                      defer_instr_bytes=defer_instr_bytes)
     names = list(op.buffers)
     ref, _ = interp.run(an, grid, bufs)
     g0, h0, _ = gpu_run(prog, names, grid, bufs, {})
@@ -226,3 +227,33 @@ def test_c1_gather_resume_nested():
     vecs = configs.c1_random_site_vectors(64, seed=11)
     scheds = [[[k] * 4] for k in range(0, 24, 2)] + [[v, v // 2] for v in vecs[:32]]
     check(cfg["ir"], 1, cfg["buffers"], scheds, flags=7 | 128)
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_osrb_smem_slots(seed):
+    """CTXB_OSRB_SMEM: the same plans with OSRB backups in per-warp shared
+    memory slots (the paper's LDS tier); poisoned forced and
+    nested preemption bit-exact, headers = oracle.  Seed 0 is the paper's
+    Fig. 5 OSRB example; the others are random loop programs."""
+    import json
+    import os
+    if seed == 0:
+        g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "fig5.json")))
+        op = ir.parse(g["ir"])
+        r = np.random.default_rng(3)
+        bufs = {b: (r.integers(0, 64, 64, dtype=np.uint32) if k == "ro" else np.zeros(64, np.uint32))
+                for b, k in op.buffers.items()}
+        prog, an = check(g["ir"], 1, bufs, [[[k]] for k in range(len(op.instrs))], runtime_flags=_cb().OSRB_SMEM)
+    else:
+        txt, size = random_program(1100 + seed, loop=True, n_body=12)
+        op = ir.parse(txt)
+        grid = 2
+        nout = op.nv - 1 + op.ns - 1
+        bufs = random_buffers(seed, op.block, grid, size, nout)
+        r = np.random.default_rng(seed)
+        nw = grid * op.nwarps
+        scheds = [[r.integers(0, 60, nw).astype(np.uint32), r.integers(0, 20, nw).astype(np.uint32)]
+                  for _ in range(4)]
+        prog, an = check(txt, grid, bufs, scheds, runtime_flags=_cb().OSRB_SMEM)
+    if an.backups:
+        assert "BKS[warp]" in prog.source
