@@ -133,6 +133,11 @@ extern "C" {
                              register (4 B per backup per thread); every lane
                              stores the warp-uniform value, each reads its own
                              write.  Plans and bytes unchanged               */
+#define CTXB_OSRB_LANES 4096u /* codegen: OSRB backup j lives in lane j % 32 of one
+                             register per 32 backups (the paper's VGPR-lane
+                             tier), read back with a warp shuffle in the
+                             (converged) preemption routine.  Exclusive with
+                             CTXB_OSRB_SMEM (_INVALID_ARG).  Plans unchanged  */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */

@@ -440,7 +440,7 @@ int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb
   if (!ir_text || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   *out = nullptr;
   ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0};
-  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 4095 || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
+  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 8191 || ((o.flags & 2048u) && (o.flags & 4096u)) || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
     return fail(CTXB_E_INVALID_ARG, "bad options");
   std::unique_ptr<ctxb_program> p(new ctxb_program);
   p->opt = Options{o.flags, o.mode, o.poll_policy, o.poll_every ? o.poll_every : 8, o.debug,

@@ -189,3 +189,19 @@ def test_osrb_smem_slots_generate_and_compile():
     m = s.backups[0]
     assert f"BKS[warp][0] = " in s.source and f"u32 bk{m} " not in s.source
     assert f"u32 bk{m} = 0u;" in base.source
+
+
+def test_osrb_lane_slots_generate_and_compile():
+    """CTXB_OSRB_LANES: backup j in lane j of one register, read by a shuffle
+    that every lane executes (hoisted out of the lane-select of the scalar
+    store); exclusive with CTXB_OSRB_SMEM."""
+    txt = configs.c4a_ir(1 << 14)
+    s = cb.Program(txt, flags=cb.ALL | cb.OSRB_LANES, poll_policy=cb.POLL_EXPLICIT)
+    assert s.info["compiled"] == 1 and s.backups
+    src = s.source
+    assert "BKV0 = lane == 0u ? " in src
+    for line in src.split("\n"):
+        if "__shfl_sync(0xffffffffu, BKV" in line:
+            assert "if (lane ==" not in line, line
+    with pytest.raises(cb.CtxbError):
+        cb.Program(txt, flags=cb.ALL | cb.OSRB_LANES | cb.OSRB_SMEM, debug=cb.DEBUG_NO_COMPILE)

@@ -69,10 +69,10 @@ def test_c3_small_forced_rank_resume():
     assert all(an.plans[c].p == c for c in an.sites)
 
 
-@pytest.mark.parametrize("smem", [False, True])
-def test_c4a_small_forced(smem):
+@pytest.mark.parametrize("slot", [0, 2048, 4096])   # register, CTXB_OSRB_SMEM, CTXB_OSRB_LANES
+def test_c4a_small_forced(slot):
     cfg = configs.c4a(1 << 14, grid=2)
-    an = forced_parity(cfg, 2, 3, 4, prog_flags=2048 if smem else 0)   # 2048 = CTXB_OSRB_SMEM
+    an = forced_parity(cfg, 2, 3, 4, prog_flags=slot)
     assert an.backups, "C4a must select an OSRB backup"
 
 

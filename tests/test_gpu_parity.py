@@ -229,12 +229,15 @@ def test_c1_gather_resume_nested():
     check(cfg["ir"], 1, cfg["buffers"], scheds, flags=7 | 128)
 
 
+@pytest.mark.parametrize("slot", ["smem", "lanes"])
 @pytest.mark.parametrize("seed", range(8))
-def test_osrb_smem_slots(seed):
-    """CTXB_OSRB_SMEM: the same plans with OSRB backups in per-warp shared
-    memory slots (the paper's LDS tier); poisoned forced and
-    nested preemption bit-exact, headers = oracle.  Seed 0 is the paper's
-    Fig. 5 OSRB example; the others are random loop programs."""
+def test_osrb_smem_slots(seed, slot):
+    """CTXB_OSRB_SMEM / CTXB_OSRB_LANES: the same plans with OSRB backups in
+    per-warp shared-memory slots (the paper's LDS tier) or in the lanes of one
+    register (the VGPR-lane tier); poisoned forced and nested
+    preemption bit-exact, headers = oracle.  Seed 0 is the paper's Fig. 5
+    OSRB example; the others are random loop programs."""
+    rf = _cb().OSRB_SMEM if slot == "smem" else _cb().OSRB_LANES
     import json
     import os
     if seed == 0:
@@ -243,7 +246,7 @@ def test_osrb_smem_slots(seed):
         r = np.random.default_rng(3)
         bufs = {b: (r.integers(0, 64, 64, dtype=np.uint32) if k == "ro" else np.zeros(64, np.uint32))
                 for b, k in op.buffers.items()}
-        prog, an = check(g["ir"], 1, bufs, [[[k]] for k in range(len(op.instrs))], runtime_flags=_cb().OSRB_SMEM)
+        prog, an = check(g["ir"], 1, bufs, [[[k]] for k in range(len(op.instrs))], runtime_flags=rf)
     else:
         txt, size = random_program(1100 + seed, loop=True, n_body=12)
         op = ir.parse(txt)
@@ -254,6 +257,6 @@ def test_osrb_smem_slots(seed):
         nw = grid * op.nwarps
         scheds = [[r.integers(0, 60, nw).astype(np.uint32), r.integers(0, 20, nw).astype(np.uint32)]
                   for _ in range(4)]
-        prog, an = check(txt, grid, bufs, scheds, runtime_flags=_cb().OSRB_SMEM)
+        prog, an = check(txt, grid, bufs, scheds, runtime_flags=rf)
     if an.backups:
-        assert "BKS[warp]" in prog.source
+        assert ("BKS[warp]" if slot == "smem" else "__shfl_sync(0xffffffffu, BKV0") in prog.source

@@ -21,7 +21,7 @@ def main():
     s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
     rows = ["| OSRB slot | regs | kernel ms (median of 7) | routines µs p50 | resume µs p50 (gathered) | preempted |",
             "|---|---|---|---|---|---|"]
-    for name, fl in (("register", 0), ("shared memory", cb.OSRB_SMEM)):
+    for name, fl in (("register", 0), ("shared memory", cb.OSRB_SMEM), ("register lanes", cb.OSRB_LANES)):
         prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT,
                           flags=cb.ALL | cb.SYNC_POLL | cb.GATHER_RESUME | fl)
         bps, nsm = prog.occupancy()
