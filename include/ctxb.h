@@ -348,6 +348,9 @@ int ctxb_read_headers(const ctxb_run* run, uint32_t* host_out, uint64_t n_words)
  * t_site_reached} (4 u64 per warp). */
 int ctxb_read_stamps(const ctxb_run* run, uint64_t* host_out, uint64_t n_words);
 
+/* Release the run handle; its device resources return to the program's pool.
+ * A launch that is still running is waited for first (not preempted).  The
+ * caller's buffers and context buffer are not freed (caller-owned). */
 int ctxb_run_destroy(ctxb_run* run);
 
 /* Header `state` values. */

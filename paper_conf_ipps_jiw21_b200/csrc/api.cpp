@@ -140,6 +140,9 @@ struct ctxb_run {
   }
   ~ctxb_run() {
     if (flag && prog) {   // return the resources to the program's pool
+      // a launch still running keeps its flag / stamps: let it finish first
+      // (disarming would otherwise preempt it)
+      if (state == RUN_RUNNING) driver().cuStreamSynchronize(stream);
       std::lock_guard<std::mutex> g(prog->mu);
       disarm();
       if (reset_pending) driver().cuEventSynchronize(evr);   // the flag is 0 again before it is reused
