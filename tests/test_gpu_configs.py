@@ -320,3 +320,37 @@ def test_statless_preempt_settles_lazily(armed):
         torch.cuda.synchronize()
         assert torch.equal(bufs[1], ref)
     assert npre > 0
+
+
+def test_destroy_running_armed_run_completes():
+    """Dropping a run handle while its (armed) launch runs waits for the launch
+    instead of firing the armed signal into it: the output is complete, and the
+    pooled resources serve the next run, which preempts and resumes bit-exact."""
+    import torch
+    cb = _cb()
+    cfg = configs.c3()
+    X = to_dev(cfg["buffers"]["X"])
+    Y = torch.zeros(cfg["W"] * cfg["H"], dtype=torch.int32, device="cuda")
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | cb.ARMED_SIGNAL)
+    bps, nsm = prog.occupancy()
+    grid = bps * nsm
+    ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
+    run = prog.launch(grid, [X, Y], [], ctx, s)
+    assert run.wait()
+    ref = Y.clone()
+    Y.zero_()
+    torch.cuda.synchronize()
+    run = prog.launch(grid, [X, Y], [], ctx, s)
+    del run                                    # still running: destroy waits, no preemption
+    torch.cuda.synchronize()
+    assert torch.equal(Y, ref)
+    Y.zero_()
+    torch.cuda.synchronize()
+    run = prog.launch(grid, [X, Y], [], ctx, s)
+    st = run.preempt(ctrl)
+    if st["warps_preempted"]:
+        run.resume(s)
+    assert run.wait()
+    torch.cuda.synchronize()
+    assert torch.equal(Y, ref)
