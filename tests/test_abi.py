@@ -158,7 +158,7 @@ def test_armed_signal_is_runtime_only():
                        debug=cb.DEBUG_NO_COMPILE)
     assert armed.source == base.source
     with pytest.raises(cb.CtxbError):
-        cb.Program(txt, flags=4096, debug=cb.DEBUG_NO_COMPILE)
+        cb.Program(txt, flags=1 << 20, debug=cb.DEBUG_NO_COMPILE)
 
 
 @pytest.mark.parametrize("flags", [cb.ALL, cb.ALL | cb.EXACT, cb.ALL | cb.RANK_RESUME | cb.PRUNE])
