@@ -130,9 +130,10 @@ extern "C" {
 #define CTXB_OSRB_SMEM  2048u /* codegen: OSRB backups live in a
                              per-warp shared-memory slot (the paper's LDS
                              tier: 4 B per backup per warp) instead of a
-                             register (4 B per backup per thread); every lane
-                             stores the warp-uniform value, each reads its own
-                             write.  Plans and bytes unchanged               */
+                             register (4 B per backup per thread); lane 0
+                             stores the warp-uniform value, the preemption
+                             routine reads it after __syncwarp().  Plans and
+                             bytes unchanged                                  */
 #define CTXB_OSRB_LANES 4096u /* codegen: OSRB backup j lives in lane j % 32 of one
                              register per 32 backups (the paper's VGPR-lane
                              tier), read back with a warp shuffle in the

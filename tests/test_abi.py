@@ -187,7 +187,8 @@ def test_osrb_smem_slots_generate_and_compile():
     assert s.info["compiled"] == 1 and s.backups == base.backups and s.backups
     assert [s.plan_text(k) for k in range(s.num_sites)] == [base.plan_text(k) for k in range(base.num_sites)]
     m = s.backups[0]
-    assert f"BKS[warp][0] = " in s.source and f"u32 bk{m} " not in s.source
+    assert "if (lane == 0u) BKS[warp][0] = " in s.source and "__syncwarp(); goto SAVE_SH_" in s.source
+    assert f"u32 bk{m} " not in s.source
     assert f"u32 bk{m} = 0u;" in base.source
 
 
