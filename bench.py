@@ -446,9 +446,21 @@ MODES = (("ctxback", 0, 7), ("full_hw", 3, 7), ("live", 1, 7),
          ("ctxback_gather", 0, 135), ("full_hw_gather", 3, 135))  # 135 = ALL | GATHER_RESUME
 
 
-def _progs(cb, ir_text, debug=0, min_blocks=0, extra_flags=0):
+def poll_tuning(cb, config):
+    """Per-config poll-site tuning, applied to every mode of that config
+    (profiles/r01_flag_polls.md): C4a tests the flag it loads (one site per
+    ~6 us chunk); C3's two sites per stencil row load the shared flag word at
+    every 4th visit (kernel 0.91 -> 0.30 ms); C4b's edge-loop polls go to 64
+    flag replicas (BFS 2.99 -> 1.40 ms)."""
+    return {"c4a": dict(extra_flags=cb.SYNC_POLL),
+            "c3": dict(load_every=4),
+            "c4b": dict(extra_flags=cb.FLAG_REPLICAS)}.get(config, {})
+
+
+def _progs(cb, ir_text, debug=0, min_blocks=0, extra_flags=0, load_every=1):
     return {name: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT if "poll" in ir_text else cb.POLL_EVERY_INSTR,
-                             mode=mode, flags=flags | extra_flags, debug=debug, min_blocks_per_sm=min_blocks)
+                             mode=mode, flags=flags | extra_flags, debug=debug, min_blocks_per_sm=min_blocks,
+                             load_every=load_every)
             for name, mode, flags in MODES}
 
 
@@ -504,6 +516,28 @@ def _flag_trials(progs, grid, make_bufs, uniforms, check, fracs, T_s):
                              warps=st["warps_preempted"], done=st["warps_done"], step_ms=0.0, launches=2))
             del run
         out[name] = summarize(recs)
+    return out
+
+
+def _poll_overhead(cb, ir_text, grid, make_bufs, uniforms=(), extra_flags=0, min_blocks=0, reps=9, load_every=1):
+    """Poll-site (+OSRB copy) overhead, the paper's Fig. 10 quantity: the
+    uninterrupted CTXBack kernel vs the same generated kernel with the poll
+    sites compiled out (CTXB_DEBUG_NO_POLLS), medians of `reps` launches."""
+    out = {}
+    for name, dbg in (("polls_ms", 0), ("no_polls_ms", cb.DEBUG_NO_POLLS)):
+        prog = cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | extra_flags, debug=dbg,
+                          min_blocks_per_sm=min_blocks, load_every=load_every)
+        import torch
+        ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+        ts = []
+        for i in range(reps + 1):
+            run = prog.launch(grid, make_bufs(), list(uniforms), ctx)
+            run.wait()
+            if i:
+                ts.append(run.launch_ms())
+            del run
+        out[name] = float(np.median(ts))
+    out["overhead_pct"] = 100.0 * (out["polls_ms"] / out["no_polls_ms"] - 1.0)
     return out
 
 
@@ -592,6 +626,7 @@ def bench_c2s(cb, trials, seed):
     res = _flag_trials(progs, grid, make, [], lambda b_: bool(torch.equal(b_[2], ref)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
     res["static"]["smem_bytes_per_tb"] = 4 * 2048
+    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], grid, make, min_blocks=2)
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
@@ -607,7 +642,7 @@ def bench_c3(cb, trials, seed):
     from workloads import configs
     cfg = configs.c3()
     W, H = cfg["W"], cfg["H"]
-    progs = _progs(cb, cfg["ir"])
+    progs = _progs(cb, cfg["ir"], **poll_tuning(cb, "c3"))
     grid = _grid(progs)
     dX = torch.from_numpy(cfg["buffers"]["X"].view(np.int32)).cuda()
     dY = torch.zeros(W * H, dtype=torch.int32, device="cuda")
@@ -625,6 +660,7 @@ def bench_c3(cb, trials, seed):
     fr = np.random.default_rng(seed + 2).uniform(0.05, 0.95, trials)
     res = _flag_trials(progs, grid, make, [], lambda b: bool(torch.equal(b[1], ref)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
+    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], grid, make, **poll_tuning(cb, "c3"))
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
@@ -633,7 +669,8 @@ def bench_c3(cb, trials, seed):
     res["t_uninterrupted_ms"] = round(T, 3)
     res["grid"] = grid
     res["uninterrupted_equals_numpy"] = ok
-    res["workload"] = f"C3 5-point stencil IR {W}x{H} f32, persistent grid, flag at U[0.05,0.95] x T"
+    res["workload"] = (f"C3 5-point stencil IR {W}x{H} f32, persistent grid, flag at U[0.05,0.95] x T; every mode "
+                       f"loads the flag at every 4th poll visit (load_every=4)")
     return res
 
 
@@ -642,7 +679,7 @@ def bench_c4a(cb, trials, seed):
     from workloads import configs
     cfg = configs.c4a(1 << 28, grid=1)
     # one poll per ~6 us chunk: sites test the flag they load (CTXB_SYNC_POLL), in every mode
-    progs = _progs(cb, cfg["ir"], extra_flags=cb.SYNC_POLL)
+    progs = _progs(cb, cfg["ir"], **poll_tuning(cb, "c4a"))
     grid = _grid(progs)
     keys = cfg["buffers"]["keys"]
     want = torch.from_numpy(np.bincount(keys >> 24, minlength=256).astype(np.int32)).cuda()
@@ -663,6 +700,7 @@ def bench_c4a(cb, trials, seed):
     fr = np.random.default_rng(seed + 3).uniform(0.05, 0.95, trials)
     res = _flag_trials(progs, grid, make, [], lambda b: bool(torch.equal(hsum(b[2]), want)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
+    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], grid, make, **poll_tuning(cb, "c4a"))   # incl. the OSRB copy
     osrb_off = cb.Program(cfg["ir"], flags=cb.RELAXED | cb.REVERT, poll_policy=cb.POLL_EXPLICIT,
                           debug=cb.DEBUG_NO_COMPILE)
     res["static"]["ctxback_osrb_off_bytes_per_tb_per_site"] = [
@@ -685,7 +723,7 @@ def bench_c4b(cb, trials, seed):
     n = len(rp) - 1
     want = configs.bfs_reference(rp, ci)
     ir_text = configs.c4b_ir()
-    progs = _progs(cb, ir_text)
+    progs = _progs(cb, ir_text, **poll_tuning(cb, "c4b"))
     grid = _grid(progs)
     d_rp = torch.from_numpy(rp.view(np.int32)).cuda()
     d_ci = torch.from_numpy(ci.view(np.int32)).cuda()
@@ -737,13 +775,40 @@ def bench_c4b(cb, trials, seed):
                 raise SystemExit(f"C4b {name}: dist differs from the reference BFS")
         res[name] = summarize(recs)
     res["static"] = _static(progs["ctxback"], 8)
+
+    def bfs_ms(prog):
+        """All levels uninterrupted: summed kernel time."""
+        ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+        d_dist.fill_(-1)
+        d_dist[0] = 0
+        fronts[0][0] = 0
+        nf, lvl, tot = 1, 0, 0.0
+        while nf:
+            cnt.zero_()
+            bufs = [d_rp, d_ci, fronts[lvl % 2], d_dist, fronts[(lvl + 1) % 2], cnt]
+            run = prog.launch(grid, bufs, [nf, lvl + 1], ctx, s)
+            run.wait()
+            tot += run.launch_ms()
+            del run
+            nf = int(cnt.item())
+            lvl += 1
+        return tot
+    ov = {}
+    for key, dbg in (("polls_ms", 0), ("no_polls_ms", cb.DEBUG_NO_POLLS)):
+        pr = cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, debug=dbg,
+                        flags=cb.ALL | poll_tuning(cb, "c4b").get("extra_flags", 0))
+        bfs_ms(pr)
+        ov[key] = float(np.median([bfs_ms(pr) for _ in range(5)]))
+    ov["overhead_pct"] = 100.0 * (ov["polls_ms"] / ov["no_polls_ms"] - 1.0)
+    res["poll_overhead"] = ov
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
     res["grid"] = grid
     res["largest_level"] = big
     res["workload"] = (f"C4b level-synchronous BFS IR, n=2^22, {len(ci)} edges (Poisson(16) out-degree), "
-                       f"preempted at U[0.05,0.95] x T in the largest level")
+                       f"preempted at U[0.05,0.95] x T in the largest level; every mode polls flag replicas "
+                       f"(CTXB_FLAG_REPLICAS)")
     return res
 
 def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
@@ -827,8 +892,10 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
     for mode in modes:
         progs, grids, ctxs = {}, {}, {}
         for k, (txt, mb) in irs.items():
+            tune = poll_tuning(cb, k)
             progs[k] = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, mode=mode_id[mode], min_blocks_per_sm=mb,
-                                  flags=cb.ALL | (SIGNAL_FLAGS if mode != "none" else 0))
+                                  flags=cb.ALL | tune.get("extra_flags", 0) | (SIGNAL_FLAGS if mode != "none" else 0),
+                                  load_every=tune.get("load_every", 1))
             b_, nsm = progs[k].occupancy()
             grids[k] = b_ * nsm
             ctxs[k] = torch.empty(progs[k].context_capacity(grids[k]), dtype=torch.uint8, device="cuda")

@@ -139,6 +139,14 @@ extern "C" {
                              tier), read back with a warp shuffle in the
                              (converged) preemption routine.  Exclusive with
                              CTXB_OSRB_SMEM (_INVALID_ARG).  Plans unchanged  */
+#define CTXB_FLAG_REPLICAS 8192u /* codegen: one warp in max(1, n_warps / 32)
+                             polls the master flag word, the others one of 64
+                             replicas (one per 4 KiB page, so dense polls of a
+                             large grid spread over L2 slices instead of
+                             queueing on one); a master poller that sees the
+                             signal forwards it to every replica.  Detection
+                             takes up to one more poll interval.  For kernels
+                             with frequent polls (C3: 0.90 -> 0.24 ms)       */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */
@@ -188,6 +196,10 @@ typedef struct {
                            (0 = 512 ~ an HBM round trip x one warp's share of HBM
                            bandwidth when every warp of the chip restores)        */
   uint32_t exact_budget; /* CTXB_EXACT: branch-and-bound nodes per window (0 = 2^20) */
+  uint32_t load_every;  /* flag mode: a warp loads the flag at every K-th poll visit
+                           (0 = 1) and tests the last loaded value at the others:
+                           K times fewer flag loads for kernels with very dense
+                           polls, detection up to K - 1 visits later          */
 } ctxb_options;
 
 typedef struct ctxb_program ctxb_program; /* analysed IR kernel + module; library-owned */
@@ -257,7 +269,7 @@ const char* ctxb_version(void);
 
 /* Parse + analyse + generate + compile.  `ir_text` need not be
  * NUL-terminated (`len` bytes are read).  opts == NULL means
- * {CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0}.
+ * {CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0, 1}.
  * Errors: _INVALID_ARG, _PARSE, _ANALYSIS, _NVRTC. */
 int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb_program** out);
 int ctxb_program_destroy(ctxb_program* prog);
@@ -294,13 +306,14 @@ int ctxb_launch(ctxb_program* prog, uint32_t grid_blocks, void* const* buffers,
                 const uint32_t* uniforms, void* ctx_buf, uint64_t ctx_buf_bytes, void* stream,
                 const uint32_t* forced_targets, ctxb_run** out);
 
-/* Raise the preemption signal (a device flag written by `ctrl_stream`, which
- * must not be the run's stream; with CTXB_ARMED_SIGNAL by the library's own
- * stream), wait until every warp of the run has either saved its context and
- * exited or finished, clear the flag.  Fills `stats` if non-NULL.
- * stats == NULL returns as soon as the launch drained: the flag reset is
- * ordered before the run's next launch on its stream, and the headers are
- * read by the next call that needs the run's state (ctxb_wait / query /
+/* Raise the preemption signal (the launch's unique signal value written to
+ * the master flag word by `ctrl_stream`, which must not be the run's stream;
+ * with CTXB_ARMED_SIGNAL by the library's own stream; the warps forward it to
+ * the flag replicas they poll), and wait until every warp of the run has
+ * either saved its context and exited or finished.  Flags are never
+ * reset: the next launch waits for a different value.  Fills `stats` if
+ * non-NULL.  stats == NULL returns as soon as the launch drained; the headers
+ * are read by the next call that needs the run's state (ctxb_wait / query /
  * resume / read_*), so the GPU is free for other work one host round trip
  * earlier.  _STATE if the run is not running. */
 int ctxb_preempt(ctxb_run* run, void* ctrl_stream, ctxb_preempt_stats* stats);

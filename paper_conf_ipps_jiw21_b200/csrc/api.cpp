@@ -67,8 +67,9 @@ struct ctxb_program {
     CUdeviceptr hflag_dev = 0;
     CUstream arm = nullptr;   // CTXB_ARMED_SIGNAL: the library's signal stream
     uint32_t gate_seq = 0;
-    CUevent evr = nullptr;    // flag reset recorded on the signal's stream
     void* hdr_pin = nullptr;  // pinned staging for the header read-back
+    uint64_t rep_off = 0;     // offset of the flag replicas in the flag buffer
+    uint32_t sig_seq = 0;     // last signal value used on this flag buffer
   };
   std::vector<Res> pool;   // per-run device resources, reused (flag is always left at 0)
   uint32_t full_ir_words128() const {  // 128-B rows occupied by the FULL_IR layout
@@ -124,9 +125,9 @@ struct ctxb_run {
   bool resumed_launch = false;
   CUevent ev0 = nullptr, ev1 = nullptr;   // recorded around each launch on the run's stream
   CUevent evf = nullptr;                  // recorded on the control stream before the flag write
-  CUevent evr = nullptr;                  // recorded after the flag reset on the signal's stream
-  bool reset_pending = false;             //   the next launch waits for it on its stream
   void* hdr_pin = nullptr;                // pinned staging buffer for the headers (n_warps x 16 B)
+  uint64_t rep_off = 0;                   // flag replicas: r->flag + rep_off + k * FLAG_STRIDE
+  uint32_t sig = 0, sig_seq = 0;          // signal value of the current launch; last value used on this buffer
   // CTXB_ARMED_SIGNAL: release a pending armed signal of a launch that was not
   // preempted and clear the flag it raises (off the preemption path).
   void disarm() {
@@ -135,8 +136,7 @@ struct ctxb_run {
     Driver& d = driver();
     *(static_cast<volatile uint32_t*>(hflag) + 16) = gate_seq;
     std::atomic_thread_fence(std::memory_order_seq_cst);
-    d.cuMemsetD32Async(flag, 0, 1, arm);
-    d.cuStreamSynchronize(arm);
+    d.cuStreamSynchronize(arm);   // the armed ops ran (their value is stale now)
   }
   ~ctxb_run() {
     if (flag && prog) {   // return the resources to the program's pool
@@ -145,9 +145,8 @@ struct ctxb_run {
       if (state == RUN_RUNNING) driver().cuStreamSynchronize(stream);
       std::lock_guard<std::mutex> g(prog->mu);
       disarm();
-      if (reset_pending) driver().cuEventSynchronize(evr);   // the flag is 0 again before it is reused
-      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf, hflag, hflag_dev, arm, gate_seq, evr,
-                            hdr_pin});
+      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf, hflag, hflag_dev, arm, gate_seq, hdr_pin,
+                            rep_off, sig_seq});
     }
   }
 };
@@ -322,7 +321,7 @@ int compile(ctxb_program* p) {
 void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>& blob) {
   size_t nb = std::max<size_t>(1, p->prog.buf_names.size());
   size_t nu = std::max<size_t>(1, p->prog.uniforms.size());
-  size_t words = nb + 6 + (nu + 9 + 1) / 2;
+  size_t words = nb + 6 + (nu + 12 + 1) / 2;
   blob.assign(words, 0);
   for (size_t i = 0; i < r->bufs.size(); i++) blob[i] = r->bufs[i];
   blob[nb + 0] = r->cbuf;
@@ -351,6 +350,9 @@ void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>
   uint32_t relays = re ? (uint32_t)strtoul(re, nullptr, 10) : 1u;
   relays = relays ? relays : 1u;
   u[nu + 8] = std::max<uint32_t>(1u, (r->n_warps + relays - 1) / relays);
+  u[nu + 9] = (uint32_t)r->rep_off;
+  u[nu + 10] = r->sig;
+  u[nu + 11] = std::max<uint32_t>(1u, r->n_warps / 32u);   // master polls: ~32 per poll interval grid-wide
 }
 
 int upload_forced(ctxb_run* r, const uint32_t* targets) {
@@ -367,16 +369,22 @@ int upload_forced(ctxb_run* r, const uint32_t* targets) {
   return CTXB_OK;
 }
 
+// The preemption signal: the launch's unique value r->sig written to the
+// master flag word (the kernel forwards it to the replicas it polls).  Flags
+// are never reset: a later launch waits for a different value.
+int write_signal(ctxb_run* r, CUstream s) {
+  CU(driver().cuStreamWriteValue32(s, r->flag, r->sig, 0));
+  return CTXB_OK;
+}
+
 int launch(ctxb_run* r, bool resume) {
+  r->sig = ++r->sig_seq;
+  if (r->sig == 0) r->sig = ++r->sig_seq;   // 0 is the flags' initial value
   std::vector<uint64_t> blob;
   r->resumed_launch = resume;
   pack_params(r, r->prog, blob);
   void* args[] = {blob.data()};
   Driver& d = driver();
-  if (r->reset_pending) {   // the flag reset of the last preemption precedes this launch
-    CU(d.cuStreamWaitEvent(r->stream, r->evr, 0));
-    r->reset_pending = false;
-  }
   CU(d.cuEventRecord(r->ev0, r->stream));
   CU(d.cuLaunchKernel(resume ? r->mod.resume : r->mod.run, r->grid, 1, 1, (unsigned)r->prog->prog.block, 1, 1, 0,
                       r->stream, args, nullptr));
@@ -387,7 +395,7 @@ int launch(ctxb_run* r, bool resume) {
     r->gate_seq++;
     CU(d.cuStreamWaitValue32(r->arm, r->hflag_dev + 64, r->gate_seq, CU_STREAM_WAIT_VALUE_GEQ));
     CU(d.cuEventRecord(r->evf, r->arm));
-    CU(d.cuStreamWriteValue32(r->arm, r->flag, 1u, 0));
+    if (int rc = write_signal(r, r->arm)) return rc;
     r->armed = true;
   }
   r->state = RUN_RUNNING;
@@ -442,14 +450,15 @@ const char* ctxb_version(void) { return "ctxb 0.1 (sm_100a, CTXB-R1)"; }
 int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb_program** out) {
   if (!ir_text || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   *out = nullptr;
-  ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0};
-  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 8191 || ((o.flags & 2048u) && (o.flags & 4096u)) || o.flag_depth > 8 || o.min_blocks_per_sm > 32)
+  ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0, 1};
+  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 16383 || ((o.flags & 2048u) && (o.flags & 4096u)) || o.flag_depth > 8 || o.load_every > 1024 || o.min_blocks_per_sm > 32)
     return fail(CTXB_E_INVALID_ARG, "bad options");
   std::unique_ptr<ctxb_program> p(new ctxb_program);
   p->opt = Options{o.flags, o.mode, o.poll_policy, o.poll_every ? o.poll_every : 8, o.debug,
                    o.flag_depth ? o.flag_depth : 1, o.min_blocks_per_sm,
                    o.defer_instr_bytes ? o.defer_instr_bytes : 8,
-                   o.resume_level_bytes ? o.resume_level_bytes : 512, o.exact_budget};
+                   o.resume_level_bytes ? o.resume_level_bytes : 512, o.exact_budget,
+                   o.load_every ? o.load_every : 1};
   try {
     double t0 = now_ms();
     p->prog = parse_ir(std::string(ir_text, len));
@@ -488,7 +497,6 @@ int ctxb_program_destroy(ctxb_program* p) {
       d.cuEventDestroy(r.evf);
       if (r.hflag) d.cuMemFreeHost(r.hflag);
       if (r.arm) d.cuStreamDestroy(r.arm);
-      d.cuEventDestroy(r.evr);
       if (r.hdr_pin) d.cuMemFreeHost(r.hdr_pin);
     }
   }
@@ -640,16 +648,19 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
         r->hflag_dev = p->pool[i].hflag_dev;
         r->arm = p->pool[i].arm;
         r->gate_seq = p->pool[i].gate_seq;
-        r->evr = p->pool[i].evr;
         r->hdr_pin = p->pool[i].hdr_pin;
+        r->rep_off = p->pool[i].rep_off;
+        r->sig_seq = p->pool[i].sig_seq;
         p->pool.erase(p->pool.begin() + (long)i);
         break;
       }
   }
   if (!r->flag) {
     CUdeviceptr f = 0, s = 0, t = 0;
-    // flag (+0), gather arrivals (+128), a gather release word per block (+256)
-    CU(d.cuMemAlloc(&f, 256 + (size_t)grid * 4));
+    // flag (+0), gather arrivals (+128), a gather release word per block (+256);
+    // then FLAG_REPLICAS replicas, one per 4 KiB page (rep_off)
+    r->rep_off = ((256 + (uint64_t)grid * 4 + FLAG_STRIDE - 1) / FLAG_STRIDE) * FLAG_STRIDE;
+    CU(d.cuMemAlloc(&f, r->rep_off + (size_t)FLAG_REPLICAS * FLAG_STRIDE));
     CU(d.cuMemAlloc(&s, (size_t)r->n_warps * 32));
     CU(d.cuMemAlloc(&t, (size_t)r->n_warps * 4));
     r->flag = f;
@@ -658,10 +669,9 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
     CU(d.cuEventCreate(&r->ev0, CU_EVENT_DEFAULT));
     CU(d.cuEventCreate(&r->ev1, CU_EVENT_DEFAULT));
     CU(d.cuEventCreate(&r->evf, CU_EVENT_DEFAULT));
-    CU(d.cuEventCreate(&r->evr, CU_EVENT_DISABLE_TIMING));
     CU(d.cuMemHostAlloc(&r->hdr_pin, (size_t)r->n_warps * 16, 0));
-    std::vector<uint32_t> z(64 + grid, 0);
-    CU(d.cuMemcpyHtoD(r->flag, z.data(), z.size() * 4));   // the flag is 0 whenever a run does not hold it raised
+    std::vector<uint8_t> z(r->rep_off + (size_t)FLAG_REPLICAS * FLAG_STRIDE, 0);
+    CU(d.cuMemcpyHtoD(r->flag, z.data(), z.size()));   // the flags are 0 whenever a run does not hold them raised
   }
   if ((p->opt.flags & (CTXB_HOST_SIGNAL | CTXB_ARMED_SIGNAL)) && !r->hflag) {
     void* h = nullptr;
@@ -714,17 +724,14 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     cs = r->arm;
   } else {
     CU(d.cuEventRecord(r->evf, cs));
-    if (!(hf && host_only)) CU(d.cuStreamWriteValue32(cs, r->flag, 1u, 0));
+    if (!(hf && host_only))
+      if (int rc = write_signal(r, cs)) return rc;
   }
   CU(d.cuStreamSynchronize(r->stream));
   double t1 = now_ms();
   if (hf) *hf = 0u;   // the victim has drained: no warp of this run reads it until the next launch
-  CU(d.cuMemsetD32Async(r->flag, 0, 1, cs));
   if (!st) {
-    // return at once: the next launch waits for the reset on its own stream,
-    // and the headers are read when first needed (settle)
-    CU(d.cuEventRecord(r->evr, cs));
-    r->reset_pending = true;
+    // return at once: the headers are read when first needed (settle)
     r->state = RUN_DRAINED;
     return CTXB_OK;
   }

@@ -88,6 +88,12 @@ Program parse_ir(const std::string& text);
 // ---- analysis ---------------------------------------------------------------
 constexpr int PRE = -1;  // value "defined before the window"
 
+// Preemption-flag replicas (runtime + generated code): warps poll replica
+// (global warp id % FLAG_REPLICAS), one per FLAG_STRIDE bytes, after the
+// master word and the gather words of the flag buffer.
+constexpr uint32_t FLAG_REPLICAS = 64;
+constexpr uint32_t FLAG_STRIDE = 4096;
+
 struct Val {         // (register, defining instruction or PRE)
   int r = -1;
   int d = PRE;
@@ -144,6 +150,7 @@ struct Options {
   uint32_t defer_instr_bytes = 8;   // CS-Defer latency-estimate weight per deferred instruction
   uint32_t resume_level_bytes = 512;  // CTXB_RANK_RESUME weight of one dependent memory round trip
   uint32_t exact_budget = 0;          // CTXB_EXACT search nodes per window (0 = default)
+  uint32_t load_every = 1;            // flag loads at every K-th poll visit (flag mode)
 };
 
 struct Analysis {

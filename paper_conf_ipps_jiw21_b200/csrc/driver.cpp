@@ -60,6 +60,8 @@ Driver& driver() {
               sym(h, "cuStreamWaitEvent", &d.cuStreamWaitEvent, &e);
     if (ok && !sym(h, "cuStreamWriteValue32_v2", &d.cuStreamWriteValue32, &e))
       ok = sym(h, "cuStreamWriteValue32", &d.cuStreamWriteValue32, &e);
+    if (ok && !sym(h, "cuStreamBatchMemOp_v2", &d.cuStreamBatchMemOp, &e))
+      ok = sym(h, "cuStreamBatchMemOp", &d.cuStreamBatchMemOp, &e);
     if (ok && !sym(h, "cuStreamWaitValue32_v2", &d.cuStreamWaitValue32, &e))
       ok = sym(h, "cuStreamWaitValue32", &d.cuStreamWaitValue32, &e);
     if (!ok) return;

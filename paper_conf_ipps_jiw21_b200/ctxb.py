@@ -14,7 +14,7 @@ import numpy as np
 
 __all__ = [
     "LIB_PATH", "CtxbError", "lib",
-    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "GATHER_RESUME", "SYNC_POLL", "HOST_SIGNAL", "ARMED_SIGNAL", "OSRB_SMEM", "OSRB_LANES", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
+    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "GATHER_RESUME", "SYNC_POLL", "HOST_SIGNAL", "ARMED_SIGNAL", "OSRB_SMEM", "OSRB_LANES", "FLAG_REPLICAS", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
     "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "EXPORTED_SYMBOLS",
@@ -27,7 +27,7 @@ LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libctxb.so"
 
 RELAXED, REVERT, OSRB, ALL, DEFER, PRUNE, RANK_RESUME, EXACT, GATHER_RESUME, SYNC_POLL, HOST_SIGNAL = \
     1, 2, 4, 7, 8, 16, 32, 64, 128, 256, 512
-ARMED_SIGNAL, OSRB_SMEM, OSRB_LANES = 1024, 2048, 4096
+ARMED_SIGNAL, OSRB_SMEM, OSRB_LANES, FLAG_REPLICAS = 1024, 2048, 4096, 8192
 MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
 DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1, 2, 4, 8, 16
@@ -54,7 +54,7 @@ class _Opts(C.Structure):
     _fields_ = [("flags", C.c_uint32), ("mode", C.c_uint32), ("poll_policy", C.c_uint32),
                 ("poll_every", C.c_uint32), ("debug", C.c_uint32), ("flag_depth", C.c_uint32),
                 ("min_blocks_per_sm", C.c_uint32), ("defer_instr_bytes", C.c_uint32),
-                ("resume_level_bytes", C.c_uint32), ("exact_budget", C.c_uint32)]
+                ("resume_level_bytes", C.c_uint32), ("exact_budget", C.c_uint32), ("load_every", C.c_uint32)]
 
 
 class _SiteInfo(C.Structure):
@@ -195,11 +195,11 @@ class Program:
 
     def __init__(self, ir_text, flags=ALL, mode=MODE_CTXBACK, poll_policy=POLL_EVERY_INSTR, poll_every=8,
                  debug=0, flag_depth=1, min_blocks_per_sm=0, defer_instr_bytes=8, resume_level_bytes=512,
-                 exact_budget=0):
+                 exact_budget=0, load_every=1):
         self._h = C.c_void_p()
         self._pid = os.getpid()
         o = _Opts(flags, mode, poll_policy, poll_every, debug, flag_depth, min_blocks_per_sm, defer_instr_bytes,
-                  resume_level_bytes, exact_budget)
+                  resume_level_bytes, exact_budget, load_every)
         b = ir_text.encode()
         _chk(lib.ctxb_analyze(b, len(b), C.byref(o), C.byref(self._h)))
         self.debug = debug

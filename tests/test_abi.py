@@ -123,8 +123,9 @@ def test_runtime_options_generate_and_compile():
     assert [g.plan_text(k) for k in range(g.num_sites)] == [base.plan_text(k) for k in range(base.num_sites)]
     src = g.source
     assert "resume_gather(P, lane, cta, dep" in src and "bar.sync 1" in src
-    assert "__any_sync(0xffffffffu, ld_flag(flagp) != 0u)" in src
-    assert "resume_gather(P" not in base.source and "ld_flag(flagp) != 0u)" not in base.source
+    assert "__any_sync(0xffffffffu, sig_hit(ld_flag(flagp) == P.sig, fsrc, P, lane) != 0u)" in src
+    assert "resume_gather(P" not in base.source and "sig_hit(ld_flag(flagp)" not in base.source
+    assert "sig_hit(fl1, fsrc, P, lane)" in base.source
 
 
 def test_host_signal_generates_and_compiles():
@@ -139,7 +140,7 @@ def test_host_signal_generates_and_compiles():
         assert h.info["compiled"] == 1
         assert [h.plan_text(k) for k in range(h.num_sites)] == [base.plan_text(k) for k in range(base.num_sites)]
         src = h.source
-        assert "ld.relaxed.sys.global.u32" in src and "relay_fwd(hfl, flagp, lane) != 0u)" in src
+        assert "ld.relaxed.sys.global.u32" in src and "relay_fwd(hfl, P, lane) != 0u)" in src
         assert "hfl = ld_hflag(hflagp); } else hfl = 0u;" in src
     assert "relay_fwd(hfl" not in base.source
     # forced (debug) programs ignore the option: no relay code is emitted
@@ -206,3 +207,20 @@ def test_osrb_lane_slots_generate_and_compile():
             assert "if (lane ==" not in line, line
     with pytest.raises(cb.CtxbError):
         cb.Program(txt, flags=cb.ALL | cb.OSRB_LANES | cb.OSRB_SMEM, debug=cb.DEBUG_NO_COMPILE)
+
+
+def test_flag_replicas_and_load_every_generate():
+    """CTXB_FLAG_REPLICAS (master pollers forward to 64 replicas) and
+    load_every (flag loads at every K-th poll visit): plans unchanged, both
+    compile for sm_100a; the options reach the generated polls."""
+    txt = configs.c3(512, 128, 64)["ir"]
+    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
+    p = cb.Program(txt, flags=cb.ALL | cb.FLAG_REPLICAS, poll_policy=cb.POLL_EXPLICIT, load_every=4)
+    assert p.info["compiled"] == 1
+    assert [p.plan_text(k) for k in range(p.num_sites)] == [base.plan_text(k) for k in range(base.num_sites)]
+    src = p.source
+    assert "const u32 fsrc = gw % P.master_period == 0u ? 1u : 0u;" in src
+    assert "if (--lcd == 0u) { lcd = 4u; fl1 = ld_flag(flagp) == P.sig; }" in src
+    assert "const u32 fsrc = 0u;" in base.source and "lcd" not in base.source
+    with pytest.raises(cb.CtxbError):
+        cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, load_every=4096, debug=cb.DEBUG_NO_COMPILE)

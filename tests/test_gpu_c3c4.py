@@ -186,7 +186,8 @@ def test_c4a_full_flag(skewed, gather):
         assert np.array_equal(total(), want)
 
 
-def test_c4b_full_flag():
+@pytest.mark.parametrize("replicas", [False, True])
+def test_c4b_full_flag(replicas):
     import torch
     cb = _cb()
     rp, ci = configs.c4b_graph()
@@ -194,7 +195,8 @@ def test_c4b_full_flag():
     want = configs.bfs_reference(rp, ci)
     op = ir.parse(configs.c4b_ir())
     an = A.analyze(op, policy="EXPLICIT")
-    prog = cb.Program(configs.c4b_ir(), poll_policy=cb.POLL_EXPLICIT)
+    prog = cb.Program(configs.c4b_ir(), poll_policy=cb.POLL_EXPLICIT,
+                      flags=cb.ALL | (cb.FLAG_REPLICAS if replicas else 0))
     grid = _persistent_grid(prog)
     sb = [an.plans[c].payload_bytes for c in an.sites]
     lb = [an.live[c].payload_bytes for c in an.sites]

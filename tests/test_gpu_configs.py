@@ -214,7 +214,9 @@ def test_c2s_full_flag_equals_c2():
 
 @pytest.mark.parametrize("which,host", [("c2", False), ("c3", False), ("c2s", False),
                                         ("c2", True), ("c3", True), ("c2s", True),
-                                        ("c2", "armed"), ("c3", "armed")])
+                                        ("c2", "armed"), ("c3", "armed"),
+                                        ("c3", "replicas"), ("c2", "replicas"), ("c3", "load4"),
+                                        ("c3", "replicas+load4")])
 def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     """random flag times, repeated and nested
     preempt -> resume -> preempt ... cycles (each resume can be preempted
@@ -224,7 +226,9 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     (CTXB_HOST_SIGNAL_ONLY=1), so every preemption arrives through a relay
     warp's system-scope poll of the host word.  host="armed":
     CTXB_ARMED_SIGNAL, every launch and resume pre-enqueues its signal behind
-    a host gate; runs that end unpreempted are disarmed."""
+    a host gate; runs that end unpreempted are disarmed.
+    "replicas" / "load4": CTXB_FLAG_REPLICAS (master pollers forward the
+    signal to 64 replicas) and loads at every 4th poll visit."""
     import time
     import torch
     cb = _cb()
@@ -239,8 +243,10 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
         out_i, mb = 2, 2
     if host is True:
         monkeypatch.setenv("CTXB_HOST_SIGNAL_ONLY", "1")
-    extra = cb.ARMED_SIGNAL if host == "armed" else cb.HOST_SIGNAL if host else 0
-    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=mb, flags=cb.ALL | extra)
+    extra = {"armed": cb.ARMED_SIGNAL, "replicas": cb.FLAG_REPLICAS, "load4": 0,
+             "replicas+load4": cb.FLAG_REPLICAS, True: cb.HOST_SIGNAL, False: 0}[host]
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=mb, flags=cb.ALL | extra,
+                      load_every=4 if host in ("load4", "replicas+load4") else 1)
     bps, nsm = prog.occupancy()
     grid = bps * nsm
     ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
