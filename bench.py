@@ -170,6 +170,7 @@ class Clocks:
 # ---- the GPU arm --------------------------------------------------------------
 
 SIGNAL_FLAGS = 0   # set by gpu_arm from --signal: cb.ARMED_SIGNAL or 0
+C3_ROWS = 2        # C3 stencil rows per loop iteration (its two poll sites per iteration)
 
 
 def make_c2(cb, size, mode, debug=0, flags=None):
@@ -449,9 +450,9 @@ MODES = (("ctxback", 0, 7), ("full_hw", 3, 7), ("live", 1, 7),
 def poll_tuning(cb, config):
     """Per-config poll-site tuning, applied to every mode of that config
     (profiles/r01_flag_polls.md): C4a tests the flag it loads (one site per
-    ~6 us chunk); C3's two sites per stencil row load the shared flag word at
-    every 4th visit (kernel 0.91 -> 0.30 ms); C4b's edge-loop polls go to 64
-    flag replicas (BFS 2.99 -> 1.40 ms)."""
+    ~6 us chunk); C3 (two stencil rows per iteration, C3_ROWS) loads the
+    shared flag word at every 4th poll visit (kernel 0.93 -> 0.19 ms); C4b's
+    edge-loop polls go to 64 flag replicas (BFS 2.99 -> 1.40 ms)."""
     return {"c4a": dict(extra_flags=cb.SYNC_POLL),
             "c3": dict(load_every=4),
             "c4b": dict(extra_flags=cb.FLAG_REPLICAS)}.get(config, {})
@@ -640,7 +641,7 @@ def bench_c2s(cb, trials, seed):
 def bench_c3(cb, trials, seed):
     import torch
     from workloads import configs
-    cfg = configs.c3()
+    cfg = configs.c3(rows_per_iter=C3_ROWS)
     W, H = cfg["W"], cfg["H"]
     progs = _progs(cb, cfg["ir"], **poll_tuning(cb, "c3"))
     grid = _grid(progs)
@@ -669,8 +670,9 @@ def bench_c3(cb, trials, seed):
     res["t_uninterrupted_ms"] = round(T, 3)
     res["grid"] = grid
     res["uninterrupted_equals_numpy"] = ok
-    res["workload"] = (f"C3 5-point stencil IR {W}x{H} f32, persistent grid, flag at U[0.05,0.95] x T; every mode "
-                       f"loads the flag at every 4th poll visit (load_every=4)")
+    res["workload"] = (f"C3 5-point stencil IR {W}x{H} f32, {C3_ROWS} rows per loop iteration (poll sites in the "
+                       f"first row's sum and after the last row's advance), persistent grid, flag at U[0.05,0.95] x T; "
+                       f"every mode loads the flag at every 4th poll visit (load_every=4)")
     return res
 
 
@@ -851,7 +853,7 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
     ls_ms = e0.elapsed_time(e1)
     # ---- batch jobs (inputs + references) ----
     c2 = configs.c2()
-    c3 = configs.c3()
+    c3 = configs.c3(rows_per_iter=C3_ROWS)
     c4a = configs.c4a(1 << 28, grid=1)
     rp, ci = configs.c4b_graph()
     bfs_want = torch.from_numpy(configs.bfs_reference(rp, ci).view(np.int32)).cuda()

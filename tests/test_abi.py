@@ -224,3 +224,18 @@ def test_flag_replicas_and_load_every_generate():
     assert "const u32 fsrc = 0u;" in base.source and "lcd" not in base.source
     with pytest.raises(cb.CtxbError):
         cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, load_every=4096, debug=cb.DEBUG_NO_COMPILE)
+
+
+@pytest.mark.parametrize("rows", [2, 4])
+def test_c3_unrolled_rows_parity(rows):
+    """C3 with several stencil rows per loop iteration (the bench's C3): the
+    same two kinds of poll site, C++ plans = oracle plans, the site after the
+    advance still reverts."""
+    txt = configs.c3_ir(512, 128, 64, rows_per_iter=rows)
+    op = ir.parse(txt)
+    an = A.analyze(op, policy="EXPLICIT")
+    p = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
+    assert p.num_sites == 2
+    for k, c in enumerate(an.sites):
+        assert p.plan_text(k) == A.plan_text(op, an.plans[c])
+    assert an.plans[an.sites[1]].n_revert_pre + an.plans[an.sites[1]].n_revert_res > 0

@@ -216,7 +216,7 @@ def test_c2s_full_flag_equals_c2():
                                         ("c2", True), ("c3", True), ("c2s", True),
                                         ("c2", "armed"), ("c3", "armed"),
                                         ("c3", "replicas"), ("c2", "replicas"), ("c3", "load4"),
-                                        ("c3", "replicas+load4")])
+                                        ("c3", "replicas+load4"), ("c3r2", "load4")])
 def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     """random flag times, repeated and nested
     preempt -> resume -> preempt ... cycles (each resume can be preempted
@@ -232,8 +232,8 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     import time
     import torch
     cb = _cb()
-    if which == "c3":
-        cfg = configs.c3()
+    if which in ("c3", "c3r2"):
+        cfg = configs.c3(rows_per_iter=2 if which == "c3r2" else 1)
         bufs = [to_dev(cfg["buffers"]["X"]), torch.zeros(cfg["W"] * cfg["H"], dtype=torch.int32, device="cuda")]
         out_i, mb = 1, 0
     else:

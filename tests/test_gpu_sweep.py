@@ -29,12 +29,13 @@ def _cases():
     return {
         "c2": (configs.c2(128, 128, 64, polls="half"), 1, (), 2),
         "c3": (configs.c3(512, 128, 64), 4, (), 0),
+        "c3r2": (configs.c3(512, 128, 64, rows_per_iter=2), 4, (), 0),
         "c4a": (configs.c4a(1 << 14, grid=2), 2, (), 0),
         "c4b": (c4b, 2, ("nextf",), 0),     # frontier order is nondeterministic: compared as a multiset
     }
 
 
-@pytest.mark.parametrize("which", ["c2", "c3", "c4a", "c4b"])
+@pytest.mark.parametrize("which", ["c2", "c3", "c3r2", "c4a", "c4b"])
 def test_every_poll_visit(which):
     import paper_conf_ipps_jiw21_b200 as cb
     cfg, grid, unordered, mb = _cases()[which]

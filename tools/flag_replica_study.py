@@ -21,8 +21,8 @@ def setup(which):
         k = torch.from_numpy(cfg["buffers"]["keys"].view(np.int32)).cuda()
         st = torch.from_numpy(cfg["buffers"]["starts"].view(np.int32)).cuda()
         return cfg["ir"], lambda g: [k, st, torch.zeros(256 * g, dtype=torch.int32, device="cuda")], 0, cb.SYNC_POLL
-    if which == "c3":
-        cfg = configs.c3()
+    if which.startswith("c3"):
+        cfg = configs.c3(rows_per_iter=int(which[3:]) if which.startswith("c3r") else 1)
         x = torch.from_numpy(cfg["buffers"]["X"].view(np.int32)).cuda()
         return cfg["ir"], lambda g: [x, torch.zeros(cfg["W"] * cfg["H"], dtype=torch.int32, device="cuda")], 0, 0
     cfg = configs.c2() if which == "c2" else configs.c2s()

@@ -204,7 +204,7 @@ def bulk_ir(nvals=64, block=256):
 
 # configs[2]: "2D 5-point stencil IR kernel with loop-carried induction
 # registers (exercises instruction reverting)".
-def c3_ir(W=8192, H=8192, strip=64, polls="both"):
+def c3_ir(W=8192, H=8192, strip=64, polls="both", rows_per_iter=1):
     """y = 0.5*x + 0.125*(N + S + W + E) on interior points (f32, IR order:
     ((N + S) + W) + E, then * 0.125, then 0.5*x + that).  Thread per column,
     256 columns x `strip` rows per work item; persistent grid, item = ctaid +
@@ -212,8 +212,11 @@ def c3_ir(W=8192, H=8192, strip=64, polls="both"):
     induction registers advance (idx += W, row += 1: reversible IADDs) and the
     finished value is written behind at idx - W.  Polls: in the middle of the
     sum, and after the advance (there CTXBack reverts idx += W at resume and
-    re-executes the loads and the sum instead of saving the result)."""
-    assert W % 256 == 0 and H % strip == 0
+    re-executes the loads and the sum instead of saving the result).
+    rows_per_iter = R > 1 unrolls R rows per loop iteration and keeps the two
+    polls in its first row's sum and after its last row's advance (poll
+    density / R: the same two kinds of site)."""
+    assert W % 256 == 0 and H % strip == 0 and strip % rows_per_iter == 0
     ncb = W // 256
     items = ncb * (H // strip)
     L = [".kernel c3_stencil", ".buffer ro X", ".buffer wo Y", ".vregs 12", ".sregs 8", ".block 256"]
@@ -234,35 +237,37 @@ def c3_ir(W=8192, H=8192, strip=64, polls="both"):
     e(f"  setp.lt.u v2, v0, {W - 1}")
     e("  and v1, v1, v2")                               # interior column
     e(f"  imad v3, s3, {W}, v0")                        # idx of (row, col)
-    e(f"  mov s5, {strip}")
+    e(f"  mov s5, {strip // rows_per_iter}")
     e("rows:")
-    e("  setp.gt.u s4, s3, 0")                          # row > 0
-    e(f"  setp.lt.u s2, s3, {H - 1}")                   # row < H-1
-    e("  and s4, s4, s2")                               # interior row
-    e("  and v11, v1, s4")                              # interior point
-    e(f"  isub v4, v3, {W}")
-    e("  @v11 ldg v5, X[v4]")                           # north
-    e(f"  iadd v4, v3, {W}")
-    e("  @v11 ldg v6, X[v4]")                           # south
-    e("  isub v4, v3, 1")
-    e("  @v11 ldg v7, X[v4]")                           # west
-    e("  iadd v4, v3, 1")
-    e("  @v11 ldg v8, X[v4]")                           # east
-    e("  ldg v9, X[v3]")                                # centre
-    e("  fadd v10, v5, v6")
-    e("  fadd v10, v10, v7")
-    if polls in ("both", "mid"):
-        e("  poll")
-    e("  fadd v10, v10, v8")
-    e("  fmul v10, v10, 0f3E000000")                    # * 0.125
-    e("  fmul v9, v9, 0f3F000000")                      # 0.5 * x
-    e("  fadd v10, v9, v10")
-    e(f"  iadd v3, v3, {W}")                            # idx += W   (reversible)
-    e("  iadd s3, s3, 1")                               # row += 1   (reversible)
-    if polls in ("both", "end"):
-        e("  poll")
-    e(f"  isub v4, v3, {W}")                            # write behind at the old idx
-    e("  @v11 stg Y[v4], v10")
+    for rr in range(rows_per_iter):
+        first, last = rr == 0, rr == rows_per_iter - 1
+        e("  setp.gt.u s4, s3, 0")                          # row > 0
+        e(f"  setp.lt.u s2, s3, {H - 1}")                   # row < H-1
+        e("  and s4, s4, s2")                               # interior row
+        e("  and v11, v1, s4")                              # interior point
+        e(f"  isub v4, v3, {W}")
+        e("  @v11 ldg v5, X[v4]")                           # north
+        e(f"  iadd v4, v3, {W}")
+        e("  @v11 ldg v6, X[v4]")                           # south
+        e("  isub v4, v3, 1")
+        e("  @v11 ldg v7, X[v4]")                           # west
+        e("  iadd v4, v3, 1")
+        e("  @v11 ldg v8, X[v4]")                           # east
+        e("  ldg v9, X[v3]")                                # centre
+        e("  fadd v10, v5, v6")
+        e("  fadd v10, v10, v7")
+        if polls in ("both", "mid") and first:
+            e("  poll")
+        e("  fadd v10, v10, v8")
+        e("  fmul v10, v10, 0f3E000000")                    # * 0.125
+        e("  fmul v9, v9, 0f3F000000")                      # 0.5 * x
+        e("  fadd v10, v9, v10")
+        e(f"  iadd v3, v3, {W}")                            # idx += W   (reversible)
+        e("  iadd s3, s3, 1")                               # row += 1   (reversible)
+        if polls in ("both", "end") and last:
+            e("  poll")
+        e(f"  isub v4, v3, {W}")                            # write behind at the old idx
+        e("  @v11 stg Y[v4], v10")
     e("  isub s5, s5, 1")
     e("  brnz s5, rows")
     e("next:")
@@ -273,11 +278,11 @@ def c3_ir(W=8192, H=8192, strip=64, polls="both"):
     return "\n".join(L) + "\n"
 
 
-def c3(W=8192, H=8192, strip=64, polls="both"):
+def c3(W=8192, H=8192, strip=64, polls="both", rows_per_iter=1):
     r = np.random.default_rng(21)
     bufs = {"X": f32_bits(r.uniform(0.0, 1.0, W * H).astype(np.float32)),
             "Y": np.zeros(W * H, dtype=np.uint32)}
-    return dict(name="C3", ir=c3_ir(W, H, strip, polls), grid=None, buffers=bufs, uniforms={},
+    return dict(name="C3", ir=c3_ir(W, H, strip, polls, rows_per_iter), grid=None, buffers=bufs, uniforms={},
                 policy="EXPLICIT", W=W, H=H, strip=strip, min_blocks=0)
 
 
