@@ -216,7 +216,8 @@ def test_c2s_full_flag_equals_c2():
                                         ("c2", True), ("c3", True), ("c2s", True),
                                         ("c2", "armed"), ("c3", "armed"),
                                         ("c3", "replicas"), ("c2", "replicas"), ("c3", "load4"),
-                                        ("c3", "replicas+load4"), ("c3r2", "load4")])
+                                        ("c3", "replicas+load4"), ("c3r2", "load4"),
+                                        ("c3r2", "combo"), ("c2", "combo"), ("c4a", "combo"), ("c4a", False)])
 def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     """random flag times, repeated and nested
     preempt -> resume -> preempt ... cycles (each resume can be preempted
@@ -232,7 +233,11 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     import time
     import torch
     cb = _cb()
-    if which in ("c3", "c3r2"):
+    if which == "c4a":
+        cfg = configs.c4a(1 << 28, grid=1)
+        bufs = [to_dev(cfg["buffers"]["keys"]), to_dev(cfg["buffers"]["starts"]), None]
+        out_i, mb = 2, 0
+    elif which in ("c3", "c3r2"):
         cfg = configs.c3(rows_per_iter=2 if which == "c3r2" else 1)
         bufs = [to_dev(cfg["buffers"]["X"]), torch.zeros(cfg["W"] * cfg["H"], dtype=torch.int32, device="cuda")]
         out_i, mb = 1, 0
@@ -243,12 +248,19 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
         out_i, mb = 2, 2
     if host is True:
         monkeypatch.setenv("CTXB_HOST_SIGNAL_ONLY", "1")
-    extra = {"armed": cb.ARMED_SIGNAL, "replicas": cb.FLAG_REPLICAS, "load4": 0,
+    # "combo": the runtime options together (armed signal, gathered resume, flag
+    # replicas, sparse flag loads; C4a also the synchronous test and shared-memory OSRB slots)
+    combo = cb.ARMED_SIGNAL | cb.GATHER_RESUME | cb.FLAG_REPLICAS
+    if which == "c4a":
+        combo |= cb.SYNC_POLL | cb.OSRB_SMEM
+    extra = {"armed": cb.ARMED_SIGNAL, "replicas": cb.FLAG_REPLICAS, "load4": 0, "combo": combo,
              "replicas+load4": cb.FLAG_REPLICAS, True: cb.HOST_SIGNAL, False: 0}[host]
     prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=mb, flags=cb.ALL | extra,
-                      load_every=4 if host in ("load4", "replicas+load4") else 1)
+                      load_every=4 if host in ("load4", "replicas+load4", "combo") else 1)
     bps, nsm = prog.occupancy()
     grid = bps * nsm
+    if bufs[out_i] is None:
+        bufs[out_i] = torch.zeros(256 * grid, dtype=torch.int32, device="cuda")
     ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
     s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
     run = prog.launch(grid, bufs, [], ctx, s)
