@@ -54,6 +54,9 @@ extern "C" {
 #define CTXB_E_STATE            -6   /* preempt on a finished run, resume on a run that
                                         is not preempted, ...                            */
 #define CTXB_E_BUFFER_TOO_SMALL -7   /* context buffer / output buffer too small         */
+#define CTXB_E_TIMEOUT          -8   /* ctxb_preempt: no drain within env
+                                        CTXB_PREEMPT_TIMEOUT_US; the run stays running
+                                        with the signal raised                          */
 
 /* ---- options (P:34-36 three techniques; P:337 compared schemes) ---------- */
 #define CTXB_RELAXED  1u  /* relaxed flashback-point condition, Alg. 1 */
@@ -272,6 +275,8 @@ const char* ctxb_version(void);
  * {CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0, 1}.
  * Errors: _INVALID_ARG, _PARSE, _ANALYSIS, _NVRTC. */
 int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb_program** out);
+/* Release the program.  Runs that still reference it keep it alive: the last
+ * run's ctxb_run_destroy frees it (any destruction order is safe). */
 int ctxb_program_destroy(ctxb_program* prog);
 int ctxb_program_info(const ctxb_program* prog, ctxb_program_info_t* out);
 int ctxb_num_sites(const ctxb_program* prog, uint32_t* n);

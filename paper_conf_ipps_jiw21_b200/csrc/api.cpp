@@ -71,7 +71,9 @@ struct ctxb_program {
     uint64_t rep_off = 0;     // offset of the flag replicas in the flag buffer
     uint32_t sig_seq = 0;     // last signal value used on this flag buffer
   };
-  std::vector<Res> pool;   // per-run device resources, reused (flag is always left at 0)
+  std::vector<Res> pool;   // per-run device resources, reused (flags hold stale signal values only)
+  int live_runs = 0;        // runs that still reference this program
+  bool destroy_pending = false;   // ctxb_program_destroy came first: the last run frees it
   uint32_t full_ir_words128() const {  // 128-B rows occupied by the FULL_IR layout
     return (uint32_t)prog.nv + ((uint32_t)prog.ns * 4 + 127) / 128;
   }
@@ -101,6 +103,8 @@ struct ctxb_program {
 // drained; the headers are read (-> PREEMPTED / DONE) on the next call that
 // needs them (settle()).
 enum { RUN_RUNNING = 0, RUN_PREEMPTED = 1, RUN_DONE = 2, RUN_DRAINED = 3 };
+
+void free_program(ctxb_program* p);
 
 struct ctxb_run {
   ctxb_program* prog = nullptr;
@@ -139,15 +143,21 @@ struct ctxb_run {
     d.cuStreamSynchronize(arm);   // the armed ops ran (their value is stale now)
   }
   ~ctxb_run() {
-    if (flag && prog) {   // return the resources to the program's pool
-      // a launch still running keeps its flag / stamps: let it finish first
-      // (disarming would otherwise preempt it)
-      if (state == RUN_RUNNING) driver().cuStreamSynchronize(stream);
+    if (!prog) return;
+    bool last = false;
+    {
       std::lock_guard<std::mutex> g(prog->mu);
-      disarm();
-      prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf, hflag, hflag_dev, arm, gate_seq, hdr_pin,
-                            rep_off, sig_seq});
+      if (flag) {   // return the resources to the program's pool
+        // a launch still running keeps its flag / stamps: let it finish first
+        // (disarming would otherwise preempt it)
+        if (state == RUN_RUNNING) driver().cuStreamSynchronize(stream);
+        disarm();
+        prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf, hflag, hflag_dev, arm, gate_seq,
+                              hdr_pin, rep_off, sig_seq});
+      }
+      last = --prog->live_runs == 0 && prog->destroy_pending;
     }
+    if (last) free_program(prog);   // the program was destroyed while this run lived
   }
 };
 
@@ -407,6 +417,8 @@ int launch(ctxb_run* r, bool resume) {
 int collect(ctxb_run* r) {
   Driver& d = driver();
   r->disarm();
+  if (r->hflag && (r->prog->opt.flags & CTXB_HOST_SIGNAL))   // the launch ended: lower a host word left raised
+    *static_cast<volatile uint32_t*>(r->hflag) = 0u;
   r->hdr_prev.swap(r->hdr);
   r->hdr.resize((size_t)r->n_warps * 4);
   CU(d.cuMemcpyDtoHAsync(r->hdr_pin, r->cbuf, (size_t)r->n_warps * 16, r->stream));
@@ -441,6 +453,25 @@ int copy_out(const std::string& s, T* buf, size_t cap, size_t* len) {
 }
 
 }  // namespace
+
+void free_program(ctxb_program* p) {
+  Driver& d = driver();
+  if (d.ok) {
+    for (auto& [c, m] : p->mods) d.cuModuleUnload(m.mod);
+    for (auto& r : p->pool) {
+      d.cuMemFree(r.flag);
+      d.cuMemFree(r.stamps);
+      d.cuMemFree(r.forced);
+      d.cuEventDestroy(r.ev0);
+      d.cuEventDestroy(r.ev1);
+      d.cuEventDestroy(r.evf);
+      if (r.hflag) d.cuMemFreeHost(r.hflag);
+      if (r.arm) d.cuStreamDestroy(r.arm);
+      if (r.hdr_pin) d.cuMemFreeHost(r.hdr_pin);
+    }
+  }
+  delete p;
+}
 
 extern "C" {
 
@@ -485,24 +516,17 @@ int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb
 
 int ctxb_program_destroy(ctxb_program* p) {
   if (!p) return fail(CTXB_E_INVALID_ARG, "NULL program");
-  Driver& d = driver();
-  if (d.ok) {
-    for (auto& [c, m] : p->mods) d.cuModuleUnload(m.mod);
-    for (auto& r : p->pool) {
-      d.cuMemFree(r.flag);
-      d.cuMemFree(r.stamps);
-      d.cuMemFree(r.forced);
-      d.cuEventDestroy(r.ev0);
-      d.cuEventDestroy(r.ev1);
-      d.cuEventDestroy(r.evf);
-      if (r.hflag) d.cuMemFreeHost(r.hflag);
-      if (r.arm) d.cuStreamDestroy(r.arm);
-      if (r.hdr_pin) d.cuMemFreeHost(r.hdr_pin);
+  {
+    std::lock_guard<std::mutex> g(p->mu);
+    if (p->live_runs > 0) {   // freed by the last run's destructor
+      p->destroy_pending = true;
+      return CTXB_OK;
     }
   }
-  delete p;
+  free_program(p);
   return CTXB_OK;
 }
+
 
 int ctxb_program_info(const ctxb_program* p, ctxb_program_info_t* o) {
   if (!p || !o) return fail(CTXB_E_INVALID_ARG, "NULL argument");
@@ -615,6 +639,10 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
   if (rc) return rc;
   std::unique_ptr<ctxb_run> r(new ctxb_run);
   r->prog = p;
+  {
+    std::lock_guard<std::mutex> g(p->mu);
+    p->live_runs++;
+  }
   r->ctx = c;
   rc = ensure_module(p, c, &r->mod);
   if (rc) return rc;
@@ -727,7 +755,22 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     if (!(hf && host_only))
       if (int rc = write_signal(r, cs)) return rc;
   }
-  CU(d.cuStreamSynchronize(r->stream));
+  // env CTXB_PREEMPT_TIMEOUT_US > 0: give up waiting for the drain after that
+  // long (a kernel without reachable poll sites); the signal stays raised and
+  // the run stays running (ctxb_wait / ctxb_query later see how it ended)
+  const char* te = getenv("CTXB_PREEMPT_TIMEOUT_US");
+  const double tmo_us = te ? atof(te) : 0.0;
+  if (tmo_us > 0.0) {
+    for (;;) {
+      CUresult q = d.cuEventQuery(r->ev1);
+      if (q == CUDA_SUCCESS) break;
+      if (q != CUDA_ERROR_NOT_READY) return fail(CTXB_E_CUDA, "cuEventQuery: " + cu_err(q));
+      if ((now_ms() - t0) * 1e3 > tmo_us)
+        return fail(CTXB_E_TIMEOUT, "the run did not drain within CTXB_PREEMPT_TIMEOUT_US (signal left raised)");
+    }
+  } else {
+    CU(d.cuStreamSynchronize(r->stream));
+  }
   double t1 = now_ms();
   if (hf) *hf = 0u;   // the victim has drained: no warp of this run reads it until the next launch
   if (!st) {

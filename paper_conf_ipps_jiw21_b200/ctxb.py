@@ -17,7 +17,7 @@ __all__ = [
     "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "GATHER_RESUME", "SYNC_POLL", "HOST_SIGNAL", "ARMED_SIGNAL", "OSRB_SMEM", "OSRB_LANES", "FLAG_REPLICAS", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
     "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS",
-    "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "EXPORTED_SYMBOLS",
+    "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "E_TIMEOUT", "EXPORTED_SYMBOLS",
     "ctxb_analyze", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait", "ctxb_context_bytes",
     "ctxb_flag_propagation",
     "Program", "Run",
@@ -34,6 +34,7 @@ DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1
 DEBUG_FENCE_STAMPS = 32
 STATE_NONE, STATE_PREEMPTED, STATE_DONE = 0, 1, 2
 NEVER = 0xFFFFFFFF
+E_TIMEOUT = -8   # ctxb_preempt gave up waiting (env CTXB_PREEMPT_TIMEOUT_US)
 
 EXPORTED_SYMBOLS = [
     "ctxb_last_error", "ctxb_version", "ctxb_analyze", "ctxb_program_destroy", "ctxb_program_info",

@@ -372,3 +372,67 @@ def test_destroy_running_armed_run_completes():
     assert run.wait()
     torch.cuda.synchronize()
     assert torch.equal(Y, ref)
+
+
+def test_preempt_timeout_leaves_run_running(monkeypatch):
+    """CTXB_PREEMPT_TIMEOUT_US: a kernel whose poll sites are compiled out
+    cannot drain; ctxb_preempt gives up with CTXB_E_TIMEOUT, the run keeps
+    running, ctxb_wait then sees it finish, and the output is complete.  With
+    a generous timeout a normal kernel preempts and resumes bit-exact."""
+    import torch
+    cb = _cb()
+    cfg = configs.c3()
+    X = to_dev(cfg["buffers"]["X"])
+    Y = torch.zeros(cfg["W"] * cfg["H"], dtype=torch.int32, device="cuda")
+    s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
+    nopoll = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_POLLS)
+    grid = nopoll.occupancy()[0] * nopoll.occupancy()[1]
+    ctx = torch.zeros(nopoll.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    run = nopoll.launch(grid, [X, Y], [], ctx, s)
+    assert run.wait()
+    ref = Y.clone()
+    Y.zero_()
+    torch.cuda.synchronize()
+    monkeypatch.setenv("CTXB_PREEMPT_TIMEOUT_US", "50")
+    run = nopoll.launch(grid, [X, Y], [], ctx, s)
+    with pytest.raises(cb.CtxbError) as ei:
+        run.preempt(ctrl)
+    assert ei.value.code == cb.E_TIMEOUT
+    assert run.wait()                      # it ran to completion
+    torch.cuda.synchronize()
+    assert torch.equal(Y, ref)
+    monkeypatch.setenv("CTXB_PREEMPT_TIMEOUT_US", "1000000")
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT)
+    ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    Y.zero_()
+    torch.cuda.synchronize()
+    run = prog.launch(grid, [X, Y], [], ctx, s)
+    st = run.preempt(ctrl)
+    if st["warps_preempted"]:
+        run.resume(s)
+    assert run.wait()
+    torch.cuda.synchronize()
+    assert torch.equal(Y, ref)
+
+
+def test_program_destroyed_before_its_run():
+    """ctxb_program_destroy while a run still references the program defers
+    the free to the last run's destruction (any finalisation order is safe)."""
+    import gc
+    import torch
+    cb = _cb()
+    cfg = configs.c3(512, 128, 64)
+    X = to_dev(cfg["buffers"]["X"])
+    Y = torch.zeros(512 * 128, dtype=torch.int32, device="cuda")
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT)
+    ctx = torch.zeros(prog.context_capacity(4), dtype=torch.uint8, device="cuda")
+    run = prog.launch(4, [X, Y], [], ctx)
+    assert cb.lib.ctxb_program_destroy(prog._h) == 0   # the run still holds it
+    prog._h = None
+    assert run.wait()
+    del run, prog
+    gc.collect()
+    torch.cuda.synchronize()
+    p2 = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT)   # the library is still healthy
+    r2 = p2.launch(4, [X, Y], [], ctx)
+    assert r2.wait()
