@@ -147,8 +147,10 @@ extern "C" {
                              replicas (one per 4 KiB page, so dense polls of a
                              large grid spread over L2 slices instead of
                              queueing on one); a master poller that sees the
-                             signal forwards it to every replica.  Detection
-                             takes up to one more poll interval.  For kernels
+                             signal forwards it to every replica; replica
+                             pollers read the master at every 64th load (so
+                             finished master pollers cannot hide a signal).
+                             Detection takes up to one more poll interval.  For kernels
                              with frequent polls (C3: 0.90 -> 0.24 ms)       */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */

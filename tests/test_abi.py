@@ -220,7 +220,7 @@ def test_flag_replicas_and_load_every_generate():
     assert [p.plan_text(k) for k in range(p.num_sites)] == [base.plan_text(k) for k in range(base.num_sites)]
     src = p.source
     assert "const u32 fsrc = gw % P.master_period == 0u ? 1u : 0u;" in src
-    assert "if (--lcd == 0u) { lcd = 4u; fl1 = ld_flag(flagp) == P.sig; }" in src
+    assert "if (--lcd == 0u) { lcd = 4u; fl1 = ld_flag(poll_addr(flagm, flagp, mcd)) == P.sig; }" in src
     assert "const u32 fsrc = 0u;" in base.source and "lcd" not in base.source
     with pytest.raises(cb.CtxbError):
         cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, load_every=4096, debug=cb.DEBUG_NO_COMPILE)
