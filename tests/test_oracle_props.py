@@ -185,3 +185,26 @@ def test_bf3_chosen_is_lexicographic_min(seed):
         feas = [pl for pl in an.candidates[c].values() if pl is not None]
         assert an.plans[c].cost() == min(pl.cost() for pl in feas)
         assert sorted(an.candidates[c]) == list(range(an.heads[c], c + 1))
+
+
+@pytest.mark.parametrize("rows", [1, 2, 4])
+def test_c3_oracle_equals_textbook_stencil_under_preemption(rows):
+    """Pin for the C3 workload as the bench runs it (rows_per_iter = 2): the
+    oracle interpreter's output equals a plain numpy 5-point stencil in the
+    IR's f32 operation order, uninterrupted and under random nested forced
+    preemption with poisoned registers, for 1, 2 and 4 rows per iteration."""
+    from workloads import configs
+    W, H = 512, 64
+    cfg = configs.c3(W, H, 32, rows_per_iter=rows)
+    op = ir.parse(cfg["ir"])
+    an = A.analyze(op, policy="EXPLICIT")
+    grid = (W // 256) * (H // 32)
+    want = configs.c3_numpy_reference(cfg["buffers"]["X"], W, H)
+    out, _ = interp.run(an, grid, cfg["buffers"])
+    assert np.array_equal(out["Y"], want)
+    r = np.random.default_rng(40 + rows)
+    nw = grid * op.nwarps
+    for _ in range(3):
+        sched = [r.integers(0, 40 // rows, nw).astype(np.uint32), r.integers(0, 8, nw).astype(np.uint32)]
+        out, rec = interp.run(an, grid, cfg["buffers"], schedule=sched, poison_seed=rows)
+        assert rec and np.array_equal(out["Y"], want)
