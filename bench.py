@@ -1003,11 +1003,12 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
                     tp0 = time.perf_counter()
                     signalled = mode != "none" and not waiting_cnt and job.run.running()
                     if signalled:
-                        job.run.preempt(ctrl, stats=False)    # returns once drained (state read later)
+                        # raise the signal and go: the LS kernels start as the victim's blocks exit
+                        job.run.preempt_async(ctrl)
                     tp1 = time.perf_counter()
                     t_ls = time.perf_counter() - t0
                     ls_job()
-                    preempted = signalled and not job.run.finished
+                    preempted = signalled and not job.run.finished   # waits for the drain
                     hp.synchronize()
                     t_ls_done = time.perf_counter() - t0
                     st = job.run.drain_stats() if preempted else None

@@ -325,6 +325,13 @@ int ctxb_launch(ctxb_program* prog, uint32_t grid_blocks, void* const* buffers,
  * earlier.  _STATE if the run is not running. */
 int ctxb_preempt(ctxb_run* run, void* ctrl_stream, ctxb_preempt_stats* stats);
 
+/* Raise the preemption signal and return at once (no drain wait): the host
+ * can launch the latency-sensitive work right away and the block scheduler
+ * starts it as the preempted blocks exit.  The run stays running until
+ * ctxb_wait / ctxb_query observe the drain (then PREEMPTED or DONE, as after
+ * ctxb_preempt).  _STATE if the run is not running. */
+int ctxb_preempt_async(ctxb_run* run, void* ctrl_stream);
+
 /* Relaunch the same grid as a resume kernel: each preempted warp reloads its
  * context, reverts / re-executes to its site and continues; finished warps
  * exit at once.  forced_targets as in ctxb_launch.  Asynchronous.

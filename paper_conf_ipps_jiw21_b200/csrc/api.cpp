@@ -812,6 +812,28 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
   return CTXB_OK;
 }
 
+int ctxb_preempt_async(ctxb_run* r, void* ctrl) {
+  if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
+  if (r->state != RUN_RUNNING) return fail(CTXB_E_STATE, "run is not running");
+  if ((CUstream)ctrl == r->stream && ctrl != nullptr)
+    return fail(CTXB_E_INVALID_ARG, "ctrl_stream must differ from the run's stream");
+  Driver& d = driver();
+  if (r->prog->opt.flags & CTXB_HOST_SIGNAL) {   // lowered when the launch is collected
+    *static_cast<volatile uint32_t*>(r->hflag) = 1u;
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+  }
+  if (r->armed) {
+    *(static_cast<volatile uint32_t*>(r->hflag) + 16) = r->gate_seq;
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    r->armed = false;
+  } else {
+    CU(d.cuEventRecord(r->evf, (CUstream)ctrl));
+    if (int rc = write_signal(r, (CUstream)ctrl)) return rc;
+  }
+  // the run stays RUNNING: ctxb_wait / ctxb_query see it drain (PREEMPTED or DONE)
+  return CTXB_OK;
+}
+
 int ctxb_resume(ctxb_run* r, void* stream, const uint32_t* forced_targets) {
   if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
   if (int rc = settle(r)) return rc;

@@ -41,7 +41,7 @@ EXPORTED_SYMBOLS = [
     "ctxb_num_sites", "ctxb_site_info", "ctxb_backups", "ctxb_site_plan_text", "ctxb_generated_source",
     "ctxb_occupancy", "ctxb_context_capacity", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait",
     "ctxb_query", "ctxb_flag_propagation", "ctxb_launch_ms", "ctxb_resume_stats_get", "ctxb_context_bytes", "ctxb_read_headers", "ctxb_read_stamps",
-    "ctxb_run_destroy",
+    "ctxb_run_destroy", "ctxb_preempt_async",
 ]
 
 
@@ -115,6 +115,7 @@ def _load():
         "ctxb_read_headers": (I, [P, C.POINTER(U32), U64]),
         "ctxb_read_stamps": (I, [P, C.POINTER(U64), U64]),
         "ctxb_run_destroy": (I, [P]),
+        "ctxb_preempt_async": (I, [P, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -305,6 +306,11 @@ class Run:
         s = _PreStats()
         _chk(lib.ctxb_preempt(self._h, _stream(ctrl_stream), C.byref(s)))
         return {k: getattr(s, k) for k, _ in _PreStats._fields_}
+
+    def preempt_async(self, ctrl_stream):
+        """Raise the signal and return at once (ctxb_preempt_async); wait() /
+        running() / finished observe the drain."""
+        _chk(lib.ctxb_preempt_async(self._h, _stream(ctrl_stream)))
 
     def drain_stats(self):
         """Device numbers of the last preempted launch, from the headers and

@@ -295,8 +295,8 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     assert cycles >= 3 and total_pre > 0
 
 
-@pytest.mark.parametrize("armed", [False, True])
-def test_statless_preempt_settles_lazily(armed):
+@pytest.mark.parametrize("armed,use_async", [(False, False), (True, False), (False, True), (True, True)])
+def test_statless_preempt_settles_lazily(armed, use_async):
     """ctxb_preempt with NULL stats returns once drained (state settled on the
     next call): repeated nested cycles on C3 with stats=False stay bit-exact,
     drain_stats() matches the header counts, and a finished run reports done."""
@@ -324,7 +324,11 @@ def test_statless_preempt_settles_lazily(armed):
             t0 = time.perf_counter()
             while time.perf_counter() < t0 + rng.uniform(0.05, 0.3) * T:
                 pass
-            assert run.preempt(ctrl, stats=False) is None
+            if use_async:   # ctxb_preempt_async: returns at once, wait() observes the drain
+                run.preempt_async(ctrl)
+                run.wait()
+            else:
+                assert run.preempt(ctrl, stats=False) is None
             if run.finished:
                 break
             d = run.drain_stats()
