@@ -1162,6 +1162,9 @@ def gpu_arm(args):
         other, oname = (0, "memop") if SIGNAL_FLAGS else (cb.ARMED_SIGNAL, "armed")
         progs["ctxback_" + oname] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | other)
         progs["full_hw_" + oname] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | other)
+        # CTXB_DRAIN_NOTICE: the host learns "drained" from a host-memory word the last warp writes
+        progs["ctxback_notice"] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | SIGNAL_FLAGS | cb.DRAIN_NOTICE)
+        progs["full_hw_notice"] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | SIGNAL_FLAGS | cb.DRAIN_NOTICE)
     bps, nsm = progs["ctxback"].occupancy()
     for p in progs.values():
         bps = min(bps, p.occupancy()[0])
@@ -1197,7 +1200,7 @@ def gpu_arm(args):
     # ---- baselines in the same framework (same fracs) ----
     base = {}
     for k in ("full_hw", "full_ir", "live", "ctxback_gather", "full_hw_gather", "ctxback_armed", "full_hw_armed",
-              "ctxback_memop", "full_hw_memop"):
+              "ctxback_memop", "full_hw_memop", "ctxback_notice", "full_hw_notice"):
         if k in progs:
             preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_w[:1], ws)
             r = preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_t, ws)
@@ -1323,7 +1326,7 @@ def gpu_arm(args):
                             main.get("context_bytes_per_tb") else None)},
         "signal": args.signal,
         "other_signal_reduction": {k: _reduction(base, "ctxback_" + k, "full_hw_" + k)
-                                   for k in ("armed", "memop") if "ctxback_" + k in base},
+                                   for k in ("armed", "memop", "notice") if "ctxback_" + k in base},
         "poll_overhead": ovh, "bulk": bulk, "configs": extra_cfg,
         "roofline": rf, "roofline_restore": rr,
         # the victim whose polls are measured: C2's FFMA SGEMM against the FP32 ALU peak

@@ -152,6 +152,15 @@ extern "C" {
                              finished master pollers cannot hide a signal).
                              Detection takes up to one more poll interval.  For kernels
                              with frequent polls (C3: 0.90 -> 0.24 ms)       */
+#define CTXB_DRAIN_NOTICE 16384u /* codegen + runtime: the launch's last warp to
+                             exit writes its signal value to a word in mapped
+                             pinned host memory (one shared-memory count per
+                             block, one global atomic per block), and
+                             ctxb_preempt returns when it sees that word
+                             instead of the kernel's completion event: host
+                             latency -5 µs on C2, but the kernel's completion
+                             (the sysmem write is flushed at kernel end) comes
+                             ~2 µs later                      */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */

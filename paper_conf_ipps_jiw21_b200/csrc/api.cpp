@@ -70,6 +70,7 @@ struct ctxb_program {
     void* hdr_pin = nullptr;  // pinned staging for the header read-back
     uint64_t rep_off = 0;     // offset of the flag replicas in the flag buffer
     uint32_t sig_seq = 0;     // last signal value used on this flag buffer
+    uint32_t drain_total = 0; // warps counted out on this flag buffer so far (mod 2^32)
   };
   std::vector<Res> pool;   // per-run device resources, reused (flags hold stale signal values only)
   int live_runs = 0;        // runs that still reference this program
@@ -132,6 +133,7 @@ struct ctxb_run {
   void* hdr_pin = nullptr;                // pinned staging buffer for the headers (n_warps x 16 B)
   uint64_t rep_off = 0;                   // flag replicas: r->flag + rep_off + k * FLAG_STRIDE
   uint32_t sig = 0, sig_seq = 0;          // signal value of the current launch; last value used on this buffer
+  uint32_t drain_base = 0, drain_total = 0;   // exit count before this launch; after it
   // CTXB_ARMED_SIGNAL: release a pending armed signal of a launch that was not
   // preempted and clear the flag it raises (off the preemption path).
   void disarm() {
@@ -153,7 +155,7 @@ struct ctxb_run {
         if (state == RUN_RUNNING) driver().cuStreamSynchronize(stream);
         disarm();
         prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf, hflag, hflag_dev, arm, gate_seq,
-                              hdr_pin, rep_off, sig_seq});
+                              hdr_pin, rep_off, sig_seq, drain_total});
       }
       last = --prog->live_runs == 0 && prog->destroy_pending;
     }
@@ -331,7 +333,7 @@ int compile(ctxb_program* p) {
 void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>& blob) {
   size_t nb = std::max<size_t>(1, p->prog.buf_names.size());
   size_t nu = std::max<size_t>(1, p->prog.uniforms.size());
-  size_t words = nb + 6 + (nu + 12 + 1) / 2;
+  size_t words = nb + 6 + (nu + 13 + 1) / 2;
   blob.assign(words, 0);
   for (size_t i = 0; i < r->bufs.size(); i++) blob[i] = r->bufs[i];
   blob[nb + 0] = r->cbuf;
@@ -363,6 +365,7 @@ void pack_params(const ctxb_run* r, const ctxb_program* p, std::vector<uint64_t>
   u[nu + 9] = (uint32_t)r->rep_off;
   u[nu + 10] = r->sig;
   u[nu + 11] = std::max<uint32_t>(1u, r->n_warps / 32u);   // master polls: ~32 per poll interval grid-wide
+  u[nu + 12] = r->drain_base;
 }
 
 int upload_forced(ctxb_run* r, const uint32_t* targets) {
@@ -390,6 +393,8 @@ int write_signal(ctxb_run* r, CUstream s) {
 int launch(ctxb_run* r, bool resume) {
   r->sig = ++r->sig_seq;
   if (r->sig == 0) r->sig = ++r->sig_seq;   // 0 is the flags' initial value
+  r->drain_base = r->drain_total;           // every block of this launch counts out once
+  r->drain_total += r->grid;
   std::vector<uint64_t> blob;
   r->resumed_launch = resume;
   pack_params(r, r->prog, blob);
@@ -482,7 +487,7 @@ int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb
   if (!ir_text || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   *out = nullptr;
   ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0, 1};
-  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 16383 || ((o.flags & 2048u) && (o.flags & 4096u)) || o.flag_depth > 8 || o.load_every > 1024 || o.min_blocks_per_sm > 32)
+  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 32767 || ((o.flags & 2048u) && (o.flags & 4096u)) || o.flag_depth > 8 || o.load_every > 1024 || o.min_blocks_per_sm > 32)
     return fail(CTXB_E_INVALID_ARG, "bad options");
   std::unique_ptr<ctxb_program> p(new ctxb_program);
   p->opt = Options{o.flags, o.mode, o.poll_policy, o.poll_every ? o.poll_every : 8, o.debug,
@@ -679,6 +684,7 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
         r->hdr_pin = p->pool[i].hdr_pin;
         r->rep_off = p->pool[i].rep_off;
         r->sig_seq = p->pool[i].sig_seq;
+        r->drain_total = p->pool[i].drain_total;
         p->pool.erase(p->pool.begin() + (long)i);
         break;
       }
@@ -687,7 +693,8 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
     CUdeviceptr f = 0, s = 0, t = 0;
     // flag (+0), gather arrivals (+128), a gather release word per block (+256);
     // then FLAG_REPLICAS replicas, one per 4 KiB page (rep_off)
-    r->rep_off = ((256 + (uint64_t)grid * 4 + FLAG_STRIDE - 1) / FLAG_STRIDE) * FLAG_STRIDE;
+    // (+ one page for the drain-notice exit counter, just below the replicas)
+    r->rep_off = ((256 + (uint64_t)grid * 4 + FLAG_STRIDE - 1) / FLAG_STRIDE) * FLAG_STRIDE + FLAG_STRIDE;
     CU(d.cuMemAlloc(&f, r->rep_off + (size_t)FLAG_REPLICAS * FLAG_STRIDE));
     CU(d.cuMemAlloc(&s, (size_t)r->n_warps * 32));
     CU(d.cuMemAlloc(&t, (size_t)r->n_warps * 4));
@@ -701,7 +708,7 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
     std::vector<uint8_t> z(r->rep_off + (size_t)FLAG_REPLICAS * FLAG_STRIDE, 0);
     CU(d.cuMemcpyHtoD(r->flag, z.data(), z.size()));   // the flags are 0 whenever a run does not hold them raised
   }
-  if ((p->opt.flags & (CTXB_HOST_SIGNAL | CTXB_ARMED_SIGNAL)) && !r->hflag) {
+  if (!r->hflag) {   // [0] host signal word, [16] armed gate, [24] drain notice
     void* h = nullptr;
     CU(d.cuMemHostAlloc(&h, 128, CU_MEMHOSTALLOC_DEVICEMAP | CU_MEMHOSTALLOC_PORTABLE));
     memset(h, 0, 128);
@@ -760,16 +767,21 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
   // the run stays running (ctxb_wait / ctxb_query later see how it ended)
   const char* te = getenv("CTXB_PREEMPT_TIMEOUT_US");
   const double tmo_us = te ? atof(te) : 0.0;
-  if (tmo_us > 0.0) {
-    for (;;) {
+  // Drained = the last warp's drain notice (host word [24] == this launch's
+  // signal value, written over PCIe as it exits) or the launch's end event,
+  // whichever the host sees first; the event is queried every ~256 spins.
+  volatile uint32_t* drain = static_cast<volatile uint32_t*>(r->hflag) + 24;
+  const bool notice = r->prog->opt.flags & CTXB_DRAIN_NOTICE;
+  if (!notice && tmo_us <= 0.0) CU(d.cuStreamSynchronize(r->stream));
+  for (uint32_t it = 0; notice || tmo_us > 0.0; it++) {
+    if (notice && *drain == r->sig) break;
+    if ((it & 255u) == 255u) {
       CUresult q = d.cuEventQuery(r->ev1);
       if (q == CUDA_SUCCESS) break;
       if (q != CUDA_ERROR_NOT_READY) return fail(CTXB_E_CUDA, "cuEventQuery: " + cu_err(q));
-      if ((now_ms() - t0) * 1e3 > tmo_us)
+      if (tmo_us > 0.0 && (now_ms() - t0) * 1e3 > tmo_us)
         return fail(CTXB_E_TIMEOUT, "the run did not drain within CTXB_PREEMPT_TIMEOUT_US (signal left raised)");
     }
-  } else {
-    CU(d.cuStreamSynchronize(r->stream));
   }
   double t1 = now_ms();
   if (hf) *hf = 0u;   // the victim has drained: no warp of this run reads it until the next launch

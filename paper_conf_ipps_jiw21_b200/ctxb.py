@@ -14,7 +14,7 @@ import numpy as np
 
 __all__ = [
     "LIB_PATH", "CtxbError", "lib",
-    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "GATHER_RESUME", "SYNC_POLL", "HOST_SIGNAL", "ARMED_SIGNAL", "OSRB_SMEM", "OSRB_LANES", "FLAG_REPLICAS", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
+    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "GATHER_RESUME", "SYNC_POLL", "HOST_SIGNAL", "ARMED_SIGNAL", "OSRB_SMEM", "OSRB_LANES", "FLAG_REPLICAS", "DRAIN_NOTICE", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
     "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "E_TIMEOUT", "EXPORTED_SYMBOLS",
@@ -27,7 +27,7 @@ LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libctxb.so"
 
 RELAXED, REVERT, OSRB, ALL, DEFER, PRUNE, RANK_RESUME, EXACT, GATHER_RESUME, SYNC_POLL, HOST_SIGNAL = \
     1, 2, 4, 7, 8, 16, 32, 64, 128, 256, 512
-ARMED_SIGNAL, OSRB_SMEM, OSRB_LANES, FLAG_REPLICAS = 1024, 2048, 4096, 8192
+ARMED_SIGNAL, OSRB_SMEM, OSRB_LANES, FLAG_REPLICAS, DRAIN_NOTICE = 1024, 2048, 4096, 8192, 16384
 MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
 DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1, 2, 4, 8, 16

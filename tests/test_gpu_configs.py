@@ -217,7 +217,8 @@ def test_c2s_full_flag_equals_c2():
                                         ("c2", "armed"), ("c3", "armed"),
                                         ("c3", "replicas"), ("c2", "replicas"), ("c3", "load4"),
                                         ("c3", "replicas+load4"), ("c3r2", "load4"),
-                                        ("c3r2", "combo"), ("c2", "combo"), ("c4a", "combo"), ("c4a", False)])
+                                        ("c3r2", "combo"), ("c2", "combo"), ("c4a", "combo"), ("c4a", False),
+                                        ("c2", "notice"), ("c3r2", "notice"), ("c2s", "notice")])
 def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     """random flag times, repeated and nested
     preempt -> resume -> preempt ... cycles (each resume can be preempted
@@ -250,10 +251,11 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
         monkeypatch.setenv("CTXB_HOST_SIGNAL_ONLY", "1")
     # "combo": the runtime options together (armed signal, gathered resume, flag
     # replicas, sparse flag loads; C4a also the synchronous test and shared-memory OSRB slots)
-    combo = cb.ARMED_SIGNAL | cb.GATHER_RESUME | cb.FLAG_REPLICAS
+    combo = cb.ARMED_SIGNAL | cb.GATHER_RESUME | cb.FLAG_REPLICAS | cb.DRAIN_NOTICE
     if which == "c4a":
         combo |= cb.SYNC_POLL | cb.OSRB_SMEM
     extra = {"armed": cb.ARMED_SIGNAL, "replicas": cb.FLAG_REPLICAS, "load4": 0, "combo": combo,
+             "notice": cb.DRAIN_NOTICE | cb.ARMED_SIGNAL,
              "replicas+load4": cb.FLAG_REPLICAS, True: cb.HOST_SIGNAL, False: 0}[host]
     prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=mb, flags=cb.ALL | extra,
                       load_every=4 if host in ("load4", "replicas+load4", "combo") else 1)
