@@ -15,7 +15,7 @@ rounding and can be wrong, so ``ffma`` uses:
      bits equals a single RN rounding (Boldo & Melquiond, "Emulation of FMA
      and correctly rounded sums: proved algorithms using rounding to odd").
 
-Pinned by tests/test_oracle_fp32.py against exact rational arithmetic
+Pinned by tests/test_oracle_arith.py against exact rational arithmetic
 (fractions.Fraction) and glibc ``fmaf``.
 """
 import numpy as np
