@@ -32,7 +32,7 @@ from __future__ import annotations
 import numpy as np
 
 from . import fp32
-from .analysis import PRE, Analysis, smem_slice
+from .analysis import MODE_FULL, PRE, Analysis, smem_slice
 
 M32 = 0xFFFFFFFF
 NEVER = 0xFFFFFFFF
@@ -355,7 +355,12 @@ class Machine:
         return np.uint32(self.S[int(r[1:])][w])
 
     def _preempt(self, w, c):
-        plan = self.an.live[c] if self.resumed_pass[w] else self.an.plans[c]
+        # R-16: a nested preemption in the resumed BB pass uses the site's LIVE
+        # plan (registers dead at c are garbage after the resume).  FULL saves
+        # every declared register regardless of liveness (the BASELINE routine
+        # "swaps all occupied resources"), so it keeps its plan.
+        nested_live = self.resumed_pass[w] and self.an.mode != MODE_FULL
+        plan = self.an.live[c] if nested_live else self.an.plans[c]
         tmp = {}
         # at-preempt reverts, decreasing m (Alg.2 MIN_COST at_preempt; Fig 3b, 6b)
         for (v, m, kind, inputs, sups) in plan.preempt_reverts:
