@@ -256,6 +256,9 @@ typedef struct {
   uint32_t exact_fallback;             /*   greedy kept although the search completed
                                           (never expected; a consistency check)       */
   double analyze_ms, codegen_ms, compile_ms;
+  uint32_t spill_stores, spill_loads;  /* ptxas -v spill bytes of the normal kernel (0 if the
+                                          log was not produced, e.g. under ncu)     */
+  uint32_t spill_stores_resume, spill_loads_resume;   /* same for ctxb_resume      */
 } ctxb_program_info_t;
 
 typedef struct {
@@ -300,6 +303,12 @@ int ctxb_site_plan_text(const ctxb_program* prog, uint32_t site, int live, char*
                         size_t* len);
 /* The generated CUDA C++ source (same buffer convention). */
 int ctxb_generated_source(const ctxb_program* prog, char* buf, size_t cap, size_t* len);
+/* The compiled sm_100a cubin (ELF) of the program's two kernels (the normal and
+ * the resume kernel): *len = its size; copied to `buf` if cap >= *len, else
+ * _BUFFER_TOO_SMALL.  _STATE if compiled with CTXB_DEBUG_NO_COMPILE.  Lets a
+ * caller inspect the generated code with its own tools (cuobjdump -sass,
+ * --dump-resource-usage) independently of this library. */
+int ctxb_program_cubin(const ctxb_program* prog, void* buf, size_t cap, size_t* len);
 
 /* Resident blocks per SM of the generated kernels (min over the normal and the
  * resume kernel, driver occupancy calculator) and the device's SM count: a

@@ -56,6 +56,7 @@ struct ctxb_program {
   std::string src, log;
   std::vector<char> cubin;
   uint32_t num_regs = 0, regs_resume = 0;
+  uint32_t spill_st = 0, spill_ld = 0, spill_st_res = 0, spill_ld_res = 0;   // ptxas -v bytes
   double t_an = 0, t_cg = 0, t_cc = 0;
   std::mutex mu;
   std::map<CUcontext, Mod> mods;
@@ -288,6 +289,21 @@ int nvrtc_compile(ctxb_program* p, uint32_t* regs_run, uint32_t* regs_resume) {
     if (std::regex_search(tail, m, std::regex("Used ([0-9]+) registers"))) return (uint32_t)std::stoul(m[1]);
     return 0;
   };
+  // ptxas -v: "N bytes stack frame, N bytes spill stores, N bytes spill loads"
+  // after the function's "Compiling entry function" line (0 when the log is absent)
+  auto spill_of = [&](const char* fn, uint32_t* st, uint32_t* ld) {
+    *st = *ld = 0;
+    size_t at = log.find(std::string("'") + fn + "'");
+    if (at == std::string::npos) return;
+    std::smatch m;
+    std::string tail = log.substr(at);
+    if (std::regex_search(tail, m, std::regex("([0-9]+) bytes spill stores, ([0-9]+) bytes spill loads"))) {
+      *st = (uint32_t)std::stoul(m[1]);
+      *ld = (uint32_t)std::stoul(m[2]);
+    }
+  };
+  spill_of("ctxb_run", &p->spill_st, &p->spill_ld);
+  spill_of("ctxb_resume", &p->spill_st_res, &p->spill_ld_res);
   *regs_run = cubin_regcount(p->cubin, "ctxb_run");
   *regs_resume = cubin_regcount(p->cubin, "ctxb_resume");
   // the two sources must agree when the log has them
@@ -558,6 +574,19 @@ int ctxb_program_info(const ctxb_program* p, ctxb_program_info_t* o) {
   o->analyze_ms = p->t_an;
   o->codegen_ms = p->t_cg;
   o->compile_ms = p->t_cc;
+  o->spill_stores = p->spill_st;
+  o->spill_loads = p->spill_ld;
+  o->spill_stores_resume = p->spill_st_res;
+  o->spill_loads_resume = p->spill_ld_res;
+  return CTXB_OK;
+}
+
+int ctxb_program_cubin(const ctxb_program* p, void* buf, size_t cap, size_t* len) {
+  if (!p || !len) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  if (p->cubin.empty()) return fail(CTXB_E_STATE, "program was analysed with CTXB_DEBUG_NO_COMPILE");
+  *len = p->cubin.size();
+  if (!buf || cap < p->cubin.size()) return fail(CTXB_E_BUFFER_TOO_SMALL, "buffer too small");
+  memcpy(buf, p->cubin.data(), p->cubin.size());
   return CTXB_OK;
 }
 
@@ -731,11 +760,34 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
   return CTXB_OK;
 }
 
+// The signal must not be ordered behind the victim kernel, or it would arrive
+// only once the kernel has finished (and "preempt" would silently wait for
+// natural completion).  Unless the signal is pre-enqueued on the library's own
+// non-blocking stream (CTXB_ARMED_SIGNAL), reject: ctrl == the run's stream;
+// ctrl == the legacy default stream (NULL / CU_STREAM_LEGACY), which waits for
+// every blocking stream; and a blocking ctrl stream when the run itself is on
+// the legacy default stream.
+static int check_ctrl(const ctxb_run* r, void* ctrl) {
+  if (r->armed) return CTXB_OK;
+  CUstream cs = (CUstream)ctrl, rs = r->stream;
+  if (cs == rs) return fail(CTXB_E_INVALID_ARG, "ctrl_stream must differ from the run's stream");
+  if (cs == nullptr || cs == CU_STREAM_LEGACY)
+    return fail(CTXB_E_INVALID_ARG, "ctrl_stream is the legacy default stream, which is ordered behind the "
+                                    "victim kernel: pass a non-blocking stream");
+  if (rs == nullptr || rs == CU_STREAM_LEGACY) {
+    unsigned fl = 0;
+    CU(driver().cuStreamGetFlags(cs, &fl));
+    if (!(fl & CU_STREAM_NON_BLOCKING))
+      return fail(CTXB_E_INVALID_ARG, "the run is on the legacy default stream and ctrl_stream is a blocking "
+                                      "stream, so the signal would wait for the victim: use non-blocking streams");
+  }
+  return CTXB_OK;
+}
+
 int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
   if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
   if (r->state != RUN_RUNNING) return fail(CTXB_E_STATE, "run is not running");
-  if ((CUstream)ctrl == r->stream && ctrl != nullptr)
-    return fail(CTXB_E_INVALID_ARG, "ctrl_stream must differ from the run's stream");
+  if (int rc = check_ctrl(r, ctrl)) return rc;
   Driver& d = driver();
   volatile uint32_t* hf =
       (r->prog->opt.flags & CTXB_HOST_SIGNAL) ? static_cast<volatile uint32_t*>(r->hflag) : nullptr;
@@ -827,8 +879,7 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
 int ctxb_preempt_async(ctxb_run* r, void* ctrl) {
   if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
   if (r->state != RUN_RUNNING) return fail(CTXB_E_STATE, "run is not running");
-  if ((CUstream)ctrl == r->stream && ctrl != nullptr)
-    return fail(CTXB_E_INVALID_ARG, "ctrl_stream must differ from the run's stream");
+  if (int rc = check_ctrl(r, ctrl)) return rc;
   Driver& d = driver();
   if (r->prog->opt.flags & CTXB_HOST_SIGNAL) {   // lowered when the launch is collected
     *static_cast<volatile uint32_t*>(r->hflag) = 1u;

@@ -57,7 +57,8 @@ Driver& driver() {
               sym(h, "cuMemHostGetDevicePointer_v2", &d.cuMemHostGetDevicePointer, &e) &&
               sym(h, "cuStreamCreateWithPriority", &d.cuStreamCreateWithPriority, &e) &&
               sym(h, "cuCtxGetStreamPriorityRange", &d.cuCtxGetStreamPriorityRange, &e) &&
-              sym(h, "cuStreamWaitEvent", &d.cuStreamWaitEvent, &e);
+              sym(h, "cuStreamWaitEvent", &d.cuStreamWaitEvent, &e) &&
+              sym(h, "cuStreamGetFlags", &d.cuStreamGetFlags, &e);
     if (ok && !sym(h, "cuStreamWriteValue32_v2", &d.cuStreamWriteValue32, &e))
       ok = sym(h, "cuStreamWriteValue32", &d.cuStreamWriteValue32, &e);
     if (ok && !sym(h, "cuStreamBatchMemOp_v2", &d.cuStreamBatchMemOp, &e))

@@ -41,7 +41,7 @@ EXPORTED_SYMBOLS = [
     "ctxb_num_sites", "ctxb_site_info", "ctxb_backups", "ctxb_site_plan_text", "ctxb_generated_source",
     "ctxb_occupancy", "ctxb_context_capacity", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait",
     "ctxb_query", "ctxb_flag_propagation", "ctxb_launch_ms", "ctxb_resume_stats_get", "ctxb_context_bytes", "ctxb_read_headers", "ctxb_read_stamps",
-    "ctxb_run_destroy", "ctxb_preempt_async",
+    "ctxb_run_destroy", "ctxb_preempt_async", "ctxb_program_cubin",
 ]
 
 
@@ -70,7 +70,8 @@ class _ProgInfo(C.Structure):
                                           "num_regs", "compiled", "num_regs_resume", "resume_maxnreg",
                                           "n_save_stubs", "cubin_bytes", "exact_windows", "exact_truncated",
                                           "exact_improved", "exact_fallback")] + \
-               [("analyze_ms", C.c_double), ("codegen_ms", C.c_double), ("compile_ms", C.c_double)]
+               [("analyze_ms", C.c_double), ("codegen_ms", C.c_double), ("compile_ms", C.c_double)] + \
+               [(n, C.c_uint32) for n in ("spill_stores", "spill_loads", "spill_stores_resume", "spill_loads_resume")]
 
 
 class _PreStats(C.Structure):
@@ -116,6 +117,7 @@ def _load():
         "ctxb_read_stamps": (I, [P, C.POINTER(U64), U64]),
         "ctxb_run_destroy": (I, [P]),
         "ctxb_preempt_async": (I, [P, P]),
+        "ctxb_program_cubin": (I, [P, P, SZ, C.POINTER(SZ)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -252,6 +254,16 @@ class Program:
     @property
     def source(self):
         return self._text(lib.ctxb_generated_source)
+
+    def cubin(self) -> bytes:
+        """The compiled sm_100a cubin (ctxb_program_cubin)."""
+        ln = C.c_size_t()
+        rc = lib.ctxb_program_cubin(self._h, None, 0, C.byref(ln))
+        if rc not in (0, -7):
+            _chk(rc)
+        buf = C.create_string_buffer(ln.value)
+        _chk(lib.ctxb_program_cubin(self._h, buf, ln.value, C.byref(ln)))
+        return buf.raw[:ln.value]
 
     def occupancy(self):
         """(resident blocks per SM, number of SMs) -> persistent grid = product."""

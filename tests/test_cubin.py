@@ -1,0 +1,93 @@
+"""The compiled sm_100a code, inspected with the CUDA toolkit's own tools
+(no GPU needed: NVRTC compiles here).
+
+* `ctxb_program_cubin` exports the cubin; `cuobjdump --dump-resource-usage`
+  reads the same register counts as the library's ELF reader (an independent
+  read; FULL_HW's bytes, 128 x NUM_REGS per warp, rest on it);
+* the save / restore stubs move the context with 128-bit evict-first global
+  stores / loads (STG.E.EF.128 / LDG.E.EF.128),
+  and the kernels use no local memory (no STL / LDL: no spilled IR
+  register), matching the ptxas spill counters in ctxb_program_info_t.
+"""
+import os
+import re
+import shutil
+import subprocess
+import tempfile
+
+import pytest
+
+from workloads import configs
+
+CUOBJDUMP = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+pytestmark = pytest.mark.skipif(not os.path.exists(CUOBJDUMP), reason="cuobjdump not installed")
+
+
+def _cuobjdump(cubin, *args):
+    with tempfile.NamedTemporaryFile(suffix=".cubin", delete=False) as f:
+        f.write(cubin)
+        path = f.name
+    try:
+        return subprocess.run([CUOBJDUMP, *args, path], check=True, capture_output=True, text=True).stdout
+    finally:
+        os.unlink(path)
+
+
+def cuobjdump_regs(cubin):
+    """{function: REG} from `cuobjdump --dump-resource-usage`."""
+    out, fn = {}, None
+    for line in _cuobjdump(cubin, "--dump-resource-usage").splitlines():
+        m = re.match(r"\s*Function (\w+):", line)
+        if m:
+            fn = m.group(1)
+        m = re.search(r"REG:(\d+).*LOCAL:(\d+)", line)
+        if m and fn:
+            out[fn] = int(m.group(1))
+            out[fn + ".local"] = int(m.group(2))
+    return out
+
+
+def cuobjdump_sass(cubin):
+    return _cuobjdump(cubin, "-sass")
+
+
+def _cb():
+    import paper_conf_ipps_jiw21_b200 as cb
+    return cb
+
+
+@pytest.mark.parametrize("name", ["c1", "c2", "c3", "c4a", "c2_full_hw"])
+def test_regcount_matches_cuobjdump(name):
+    cb = _cb()
+    mode = cb.MODE_FULL_HW if name.endswith("full_hw") else cb.MODE_CTXBACK
+    if name == "c1":
+        prog = cb.Program(configs.c1()["ir"], debug=cb.DEBUG_FORCED, mode=mode)
+    elif name.startswith("c2"):
+        prog = cb.Program(configs.c2(256, 256, 64)["ir"], poll_policy=cb.POLL_EXPLICIT, mode=mode, min_blocks_per_sm=2)
+    elif name == "c3":
+        prog = cb.Program(configs.c3(rows_per_iter=2)["ir"], poll_policy=cb.POLL_EXPLICIT, mode=mode)
+    else:
+        prog = cb.Program(configs.c4a(1 << 14, grid=1)["ir"], poll_policy=cb.POLL_EXPLICIT, mode=mode)
+    info = prog.info
+    cub = prog.cubin()
+    assert len(cub) == info["cubin_bytes"] and cub[:4] == b"\x7fELF"
+    regs = cuobjdump_regs(cub)
+    assert regs["ctxb_run"] == info["num_regs"]
+    assert regs["ctxb_resume"] == info["num_regs_resume"]
+    # no local memory <=> no spill bytes reported by ptxas
+    assert regs["ctxb_run.local"] == 0 and info["spill_stores"] == 0 and info["spill_loads"] == 0
+    assert regs["ctxb_resume.local"] == 0 and info["spill_stores_resume"] == 0
+
+
+def test_c2_stubs_are_128bit_and_spill_free():
+    cb = _cb()
+    prog = cb.Program(configs.c2(256, 256, 64)["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=2)
+    sass = cuobjdump_sass(prog.cubin())
+    ops = re.findall(r"\b(STG|LDG|STL|LDL)(\.[A-Z0-9.]+)?", sass)
+    names = ["".join(o) for o in ops]
+    assert not any(n.startswith(("STL", "LDL")) for n in names), "local-memory traffic in the generated kernels"
+    # C2's plans save 68-70 vector values per warp: the save and restore stubs
+    # move them as 128-bit evict-first accesses (one v4 per 4 values)
+    n_st = sum(1 for n in names if n.startswith("STG") and n.endswith(".128") and ".EF" in n)
+    n_ld = sum(1 for n in names if n.startswith("LDG") and n.endswith(".128") and ".EF" in n)
+    assert n_st >= 16 and n_ld >= 16, (n_st, n_ld)

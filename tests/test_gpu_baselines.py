@@ -1,0 +1,191 @@
+"""GPU parity of the baselines every reduction is reported against (SURVEY
+§8 row a9): the same generated kernels built in
+CTXB_MODE_LIVE (save LIVE_IN(site)), CTXB_MODE_FULL (FULL_IR: every declared
+IR register) and CTXB_MODE_FULL_HW (FULL_IR padded to the compiled kernel's
+register count per thread: "all occupied resources regardless of liveness").
+
+* outputs after forced (poisoned, nested) and flag preemption are bit-exact
+  against the oracle interpreter run in the same mode (FULL_HW restores its
+  FULL_IR part; the padding words are written and read back);
+* per-warp header bytes equal the oracle's plan bytes (LIVE / FULL_IR);
+* FULL_HW header bytes equal 128 x NUM_REGS per warp, NUM_REGS read from the
+  exported cubin by `cuobjdump --dump-resource-usage` (independent of the
+  library's own ELF reader).
+"""
+import numpy as np
+import pytest
+
+from oracle import analysis as A
+from oracle import interp, ir
+from workloads import configs
+
+from gpu_helpers import gpu_run, header_records, oracle_records, to_dev
+from test_cubin import cuobjdump_regs
+
+pytestmark = pytest.mark.gpu
+
+MODES = {"live": 1, "full_ir": 2, "full_hw": 3}
+
+
+def _cb():
+    import paper_conf_ipps_jiw21_b200 as cb
+    return cb
+
+
+def hw_bytes(prog, op):
+    """FULL_HW bytes per warp: NUM_REGS x 128 B (cuobjdump), at least the
+    FULL_IR rows (vector registers + scalars packed 32 per 128 B row)."""
+    regs = cuobjdump_regs(prog.cubin())["ctxb_run"]
+    assert regs == prog.info["num_regs"]
+    rows = op.nv + (4 * op.ns + 127) // 128
+    return 128 * max(regs, rows)
+
+
+def expected_records(rec, an, mode, prog, op):
+    want = oracle_records(rec, an)
+    if mode == 3:
+        hb = hw_bytes(prog, op)
+        want = [{w: (k, live, hb) for w, (k, live, _b) in d.items()} for d in want]
+    return want
+
+
+def check_mode(txt, grid, bufs, schedules, mode, policy="EVERY_INSTR", min_blocks=0, skip=("scr",)):
+    cb = _cb()
+    op = ir.parse(txt)
+    an = A.analyze(op, policy=policy, mode=min(mode, 2))
+    pol = {"EVERY_INSTR": cb.POLL_EVERY_INSTR, "EXPLICIT": cb.POLL_EXPLICIT}[policy]
+    prog = cb.Program(txt, poll_policy=pol, mode=mode, debug=cb.DEBUG_FORCED | cb.DEBUG_POISON,
+                      min_blocks_per_sm=min_blocks)
+    names = list(op.buffers)
+    ref, _ = interp.run(an, grid, bufs)
+    g0, _h, _ = gpu_run(prog, names, grid, bufs, {})
+    for n in names:
+        if n not in skip:
+            assert np.array_equal(g0[n], ref[n]), f"uninterrupted {n} differs"
+    for sched in schedules:
+        out, rec = interp.run(an, grid, bufs, schedule=sched)
+        g, hdrs, _ = gpu_run(prog, names, grid, bufs, {}, schedule=sched)
+        for n in names:
+            if n not in skip:
+                assert np.array_equal(out[n], ref[n])
+                assert np.array_equal(g[n], ref[n]), f"{n} differs after preempt/resume ({sched})"
+        want = expected_records(rec, an, mode, prog, op)
+        assert header_records(hdrs)[:len(want)] == want
+    return prog, an
+
+
+@pytest.mark.parametrize("mode", list(MODES))
+def test_c1_every_site(mode):
+    cfg = configs.c1()
+    check_mode(cfg["ir"], 1, cfg["buffers"], [[[k] * 4] for k in range(24)], MODES[mode])
+
+
+@pytest.mark.parametrize("mode", list(MODES))
+def test_c1_random_nested(mode):
+    cfg = configs.c1()
+    vecs = configs.c1_random_site_vectors(64)
+    r = np.random.default_rng(11)
+    scheds = [[v, r.integers(0, 6, 4).astype(np.uint32)] if i % 2 else [v] for i, v in enumerate(vecs)]
+    check_mode(cfg["ir"], 1, cfg["buffers"], scheds, MODES[mode])
+
+
+@pytest.mark.parametrize("mode", list(MODES))
+def test_c2_small_forced_nested(mode):
+    M, N, K = 128, 128, 64
+    cfg = configs.c2(M, N, K)
+    r = np.random.default_rng(21)
+    visits = K // 4
+    scheds = [[r.integers(0, visits, 8).astype(np.uint32), r.integers(0, 8, 8).astype(np.uint32)] for _ in range(3)]
+    check_mode(cfg["ir"], 1, cfg["buffers"], scheds, MODES[mode], policy="EXPLICIT", min_blocks=cfg["min_blocks"])
+
+
+@pytest.mark.parametrize("mode", list(MODES))
+def test_c2_full_size_flag(mode):
+    """4096^3 on the persistent grid; flag at 30 % and 60 % of T: C bit-exact
+    with the uninterrupted run, every preempted warp's header bytes = the
+    mode's plan bytes (FULL_HW: 128 x NUM_REGS)."""
+    import time
+    import torch
+    cb = _cb()
+    cfg = configs.c2()
+    M, N = cfg["M"], cfg["N"]
+    op = ir.parse(cfg["ir"])
+    m = MODES[mode]
+    an = A.analyze(op, policy="EXPLICIT", mode=min(m, 2))
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, mode=m, min_blocks_per_sm=cfg["min_blocks"])
+    bps, nsm = prog.occupancy()
+    grid = bps * nsm
+    dA, dB = to_dev(cfg["buffers"]["A"]), to_dev(cfg["buffers"]["B"])
+    dC = torch.zeros(M * N, dtype=torch.int32, device="cuda")
+    ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
+    run = prog.launch(grid, [dA, dB, dC], [], ctx, s)
+    assert run.wait()
+    T = run.launch_ms() / 1e3
+    ref = dC.clone()
+    want = {k: (hw_bytes(prog, op) if m == 3 else an.plans[c].payload_bytes) for k, c in enumerate(an.sites)}
+    seen = 0
+    for frac in (0.3, 0.6):
+        dC.zero_()
+        torch.cuda.synchronize()
+        run = prog.launch(grid, [dA, dB, dC], [], ctx, s)
+        t0 = time.perf_counter()
+        while time.perf_counter() < t0 + frac * T:
+            pass
+        st = run.preempt(ctrl)
+        if st["warps_preempted"]:
+            h = run.headers()
+            pre = (h[:, 2] == 1) & (h[:, 3] == 1)
+            for w in np.nonzero(pre)[0]:
+                assert int(h[w, 1]) == want[int(h[w, 0]) & 0x7FFFFFFF], (w, h[w])
+            assert st["payload_bytes"] == int(h[pre, 1].astype(np.int64).sum())
+            seen += int(pre.sum())
+            run.resume(s)
+            assert run.wait()
+        torch.cuda.synchronize()
+        assert torch.equal(dC, ref), f"{mode}: C differs after preempt/resume at {frac} T"
+    assert seen > 0, "no warp was preempted"
+
+
+def test_ctrl_stream_checks():
+    """ADVICE: a signal that would be ordered behind the victim is rejected
+    (legacy default stream as ctrl; a blocking ctrl with the run on the legacy
+    default stream); the armed signal needs no ctrl stream."""
+    import ctypes
+    import torch
+    cb = _cb()
+    cfg = configs.c2()
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=cfg["min_blocks"])
+    bps, nsm = prog.occupancy()
+    grid = bps * nsm
+    dA, dB = to_dev(cfg["buffers"]["A"]), to_dev(cfg["buffers"]["B"])
+    dC = torch.zeros(cfg["M"] * cfg["N"], dtype=torch.int32, device="cuda")
+    ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    s = torch.cuda.Stream()
+    run = prog.launch(grid, [dA, dB, dC], [], ctx, s)
+    with pytest.raises(cb.CtxbError) as e:
+        run.preempt(None)
+    assert e.value.code == -1
+    with pytest.raises(cb.CtxbError):
+        run.preempt(s)
+    assert run.wait()
+    libcuda = ctypes.CDLL("libcuda.so.1")
+    hs = ctypes.c_void_p()
+    assert libcuda.cuStreamCreate(ctypes.byref(hs), 0) == 0          # a blocking stream
+    try:
+        run = prog.launch(grid, [dA, dB, dC], [], ctx, None)         # the legacy default stream
+        with pytest.raises(cb.CtxbError) as e:
+            run.preempt(hs.value)
+        assert e.value.code == -1
+        assert run.wait()
+    finally:
+        torch.cuda.synchronize()
+        libcuda.cuStreamDestroy_v2(hs)
+    armed = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=cfg["min_blocks"],
+                       flags=cb.ALL | cb.ARMED_SIGNAL)
+    ctx2 = torch.zeros(armed.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    run = armed.launch(grid, [dA, dB, dC], [], ctx2, s)
+    st = run.preempt(None)                                           # the library's own stream signals
+    if st["warps_preempted"]:
+        run.resume(s)
+    assert run.wait()
