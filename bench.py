@@ -172,7 +172,7 @@ class Clocks:
 # ---- the GPU arm --------------------------------------------------------------
 
 SIGNAL_FLAGS = 0   # set by gpu_arm from --signal: cb.ARMED_SIGNAL or 0
-C3_ROWS = 2        # C3 stencil rows per loop iteration (its two poll sites per iteration)
+C3_ROWS = 8        # C3 stencil rows per loop iteration, one (reverting) poll site per iteration (configs.BENCH_C3)
 
 
 def make_c2(cb, size, mode, debug=0, flags=None):
@@ -330,6 +330,35 @@ def bulk_bandwidth(cb, mib, reps=5):
                 save_bytes=save_bytes, restore_bytes=rest_bytes)
 
 
+def restore_floor(cb, nvals, grid, reps=9):
+    """The cold-read floor of an in-situ restore of this size on this grid:
+    the bulk IR kernel (every warp's LIVE context = `nvals` vector values,
+    saved through the generated save stub), L2 evicted, then the resume
+    kernel's restore stub reads it back with no replay.  Device span (the
+    resume time's definition: first warp entry -> last warp restored),
+    median of `reps`.  tools/restore_micro.cu measures the same floor with a
+    hand-written read kernel (profiles/r02_restore_floor.md)."""
+    import torch
+    from workloads import configs
+    prog = cb.Program(configs.bulk_ir(nvals), poll_policy=cb.POLL_EXPLICIT, mode=cb.MODE_LIVE,
+                      debug=cb.DEBUG_FORCED, min_blocks_per_sm=2)
+    nw = grid * 8
+    out = torch.zeros(256, dtype=torch.int32, device="cuda")
+    ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    s = torch.cuda.Stream()
+    spans = []
+    for i in range(reps + 1):
+        run = prog.launch(grid, [out], [], ctx, s, forced=np.zeros(nw, np.uint32))
+        assert not run.wait()
+        evict_l2(s)
+        run.resume(s, forced=np.full(nw, cb.NEVER, np.uint32))
+        assert run.wait()
+        if i:
+            spans.append(run.resume_stats()["resume_us"])
+        del run
+    return float(np.median(spans))
+
+
 def poll_overhead(cb, size, grid, bufs, reps=20):
     import torch
     out = {}
@@ -451,12 +480,12 @@ MODES = (("ctxback", 0, 7), ("full_hw", 3, 7), ("live", 1, 7),
 
 def poll_tuning(cb, config):
     """Per-config poll-site tuning, applied to every mode of that config
-    (profiles/r01_flag_polls.md): C4a tests the flag it loads (one site per
-    ~6 us chunk); C3 (two stencil rows per iteration, C3_ROWS) loads the
-    shared flag word at every 4th poll visit (kernel 0.93 -> 0.19 ms); C4b's
-    edge-loop polls go to 64 flag replicas (BFS 2.99 -> 1.40 ms)."""
+    (profiles/r01_flag_polls.md, profiles/r02_poll_placement.md): C4a tests
+    the flag it loads (one site per ~6 us chunk); C3 (configs.BENCH_C3: 8 rows
+    per iteration, the reverting site only) loads the one flag word at every
+    visit; C4b's edge-chunk polls (configs.BENCH_C4B_POLLS) go to 64 flag
+    replicas."""
     return {"c4a": dict(extra_flags=cb.SYNC_POLL),
-            "c3": dict(load_every=4),
             "c4b": dict(extra_flags=cb.FLAG_REPLICAS)}.get(config, {})
 
 
@@ -643,7 +672,7 @@ def bench_c2s(cb, trials, seed):
 def bench_c3(cb, trials, seed):
     import torch
     from workloads import configs
-    cfg = configs.c3(rows_per_iter=C3_ROWS)
+    cfg = configs.c3(**configs.BENCH_C3)
     W, H = cfg["W"], cfg["H"]
     progs = _progs(cb, cfg["ir"], **poll_tuning(cb, "c3"))
     grid = _grid(progs)
@@ -672,9 +701,8 @@ def bench_c3(cb, trials, seed):
     res["t_uninterrupted_ms"] = round(T, 3)
     res["grid"] = grid
     res["uninterrupted_equals_numpy"] = ok
-    res["workload"] = (f"C3 5-point stencil IR {W}x{H} f32, {C3_ROWS} rows per loop iteration (poll sites in the "
-                       f"first row's sum and after the last row's advance), persistent grid, flag at U[0.05,0.95] x T; "
-                       f"every mode loads the flag at every 4th poll visit (load_every=4)")
+    res["workload"] = (f"C3 5-point stencil IR {W}x{H} f32, {C3_ROWS} rows per loop iteration, one poll site after "
+                       f"the last row's advance (reverting site), persistent grid, flag at U[0.05,0.95] x T")
     return res
 
 
@@ -726,7 +754,7 @@ def bench_c4b(cb, trials, seed):
     rp, ci = configs.c4b_graph()
     n = len(rp) - 1
     want = configs.bfs_reference(rp, ci)
-    ir_text = configs.c4b_ir()
+    ir_text = configs.c4b_ir(configs.BENCH_C4B_POLLS)
     progs = _progs(cb, ir_text, **poll_tuning(cb, "c4b"))
     grid = _grid(progs)
     d_rp = torch.from_numpy(rp.view(np.int32)).cuda()
@@ -811,8 +839,8 @@ def bench_c4b(cb, trials, seed):
     res["grid"] = grid
     res["largest_level"] = big
     res["workload"] = (f"C4b level-synchronous BFS IR, n=2^22, {len(ci)} edges (Poisson(16) out-degree), "
-                       f"preempted at U[0.05,0.95] x T in the largest level; every mode polls flag replicas "
-                       f"(CTXB_FLAG_REPLICAS)")
+                       f"preempted at U[0.05,0.95] x T in the largest level; poll site before each edge chunk's "
+                       f"atomics only, every mode polls flag replicas (CTXB_FLAG_REPLICAS)")
     return res
 
 def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
@@ -855,7 +883,7 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
     ls_ms = e0.elapsed_time(e1)
     # ---- batch jobs (inputs + references) ----
     c2 = configs.c2()
-    c3 = configs.c3(rows_per_iter=C3_ROWS)
+    c3 = configs.c3(**configs.BENCH_C3)
     c4a = configs.c4a(1 << 28, grid=1)
     rp, ci = configs.c4b_graph()
     bfs_want = torch.from_numpy(configs.bfs_reference(rp, ci).view(np.int32)).cuda()
@@ -877,7 +905,7 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
     }
     hist_want = torch.from_numpy(np.bincount(c4a["buffers"]["keys"] >> 24, minlength=256).astype(np.int32)).cuda()
     irs = {"c2": (configs.c2_ir(4096, 4096, 4096, polls="iter"), 2), "c3": (c3["ir"], 0),
-           "c4a": (c4a["ir"], 0), "c4b": (configs.c4b_ir(), 0)}
+           "c4a": (c4a["ir"], 0), "c4b": (configs.c4b_ir(configs.BENCH_C4B_POLLS), 0)}
     mode_id = {"ctxback": cb.MODE_CTXBACK, "full_hw": cb.MODE_FULL_HW, "none": cb.MODE_CTXBACK}
     results = {}
     refs = {}
@@ -1217,6 +1245,14 @@ def gpu_arm(args):
         "full_hw_bytes_per_tb": nwb * 128 * progs.get("full_hw", pr).info["num_regs"],
         "num_regs": pr.info["num_regs"],
     }
+    # ---- cold-read floor of the in-situ restores (same bytes per warp, same grid, no replay) ----
+    floor = {}
+    for k, m in (("ctxback", main), ("full_hw", base.get("full_hw"))):
+        if m and m.get("context_bytes_per_tb"):
+            nv = int(round(m["context_bytes_per_tb"] / 8 / 128))
+            floor[k] = {"values_per_warp": nv, "resume_floor_us": restore_floor(cb, nv, grid),
+                        "resume_us": m["resume_us_median"]}
+            floor[k]["frac_of_floor"] = floor[k]["resume_floor_us"] / max(1e-9, m["resume_us_median"])
     # ---- poll overhead, bulk roofline ----
     ovh = poll_overhead(cb, size, grid, (dA, dB, dC))
     bulk = bulk_bandwidth(cb, args.bulk_mib)
@@ -1337,7 +1373,7 @@ def gpu_arm(args):
         "signal": args.signal,
         "other_signal_reduction": {k: _reduction(base, "ctxback_" + k, "full_hw_" + k)
                                    for k in ("armed", "memop", "notice") if "ctxback_" + k in base},
-        "poll_overhead": ovh, "bulk": bulk, "configs": extra_cfg,
+        "poll_overhead": ovh, "bulk": bulk, "configs": extra_cfg, "restore_floor": floor,
         "roofline": rf, "roofline_restore": rr,
         # the victim whose polls are measured: C2's FFMA SGEMM against the FP32 ALU peak
         # derived from unit counts and clocks (148 SMs x 128 FP32 lanes x 2 flops x max SM clock)
@@ -1374,10 +1410,12 @@ def compact_line(d, detail_path):
     fh = d["baselines"].get("full_hw", {})
     rf = {k: d["roofline"][k] for k in ("bound", "achieved", "peak", "unit", "frac", "traffic")}
     rr = {k: d["roofline_restore"][k] for k in ("bound", "achieved", "peak", "unit", "frac", "traffic")}
+    for x in (rf, rr):
+        x["achieved"], x["peak"], x["frac"] = round(x["achieved"]), round(x["peak"]), round(x["frac"], 3)
     cpu = d.get("cpu_baseline")
     if cpu:
         cpu = {"value": _r(cpu["value"], 1), "unit": cpu["unit"], "cores": cpu["cores"], "kind": "oracle",
-               "sample": "C2 IR 256^3, TB 0, 8 warps preempted at one poll visit"}
+               "sample": "C2 IR 256^3, TB0, 8 warps, 1 poll visit"}
     e = d["e2e"]
     cfgs = {}
     for k, c in d.get("configs", {}).items():
@@ -1397,27 +1435,28 @@ def compact_line(d, detail_path):
         "metric": d["metric"], "value": d["value"], "unit": d["unit"], "n_gpus": d["n_gpus"], "steps": d["steps"],
         "warmup": d["warmup"], "ms_per_step": d["ms_per_step"], "higher_is_better": False, "scaling": "weak",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": f"C2 SGEMM IR {d['config']['size']}^3 f32 (configs[1]), {d['config']['grid']}x256 "
-                               "persistent grid, flag at U[.05,.95]xT",
+        "config": {"workload": f"C2 SGEMM IR {d['config']['size']}^3 (configs[1]), {d['config']['grid']}x256 "
+                               "persistent, flag U[.05,.95]T",
                    "l2": "inputs > L2; resume L2-cold" if "cold" in d["config"]["resume_l2"] else "inputs > L2; resume warm"},
-        "value_is": "signal->drained, CUDA events, median",
         "routines_us": _r(m["latency_us_median"], 3), "resume_us": _r(m["resume_us_median"], 3),
         "context_bytes_per_tb": m.get("context_bytes_per_tb"),
         "full_hw": {"value": _r(fh.get("signal_to_drained_us_median"), 3), "routines_us": _r(fh.get("latency_us_median"), 3),
                     "resume_us": _r(fh.get("resume_us_median"), 3), "context_bytes_per_tb": fh.get("context_bytes_per_tb")},
-        "reduction_vs_full_hw_pct": {"value": d["reduction_vs_full_hw"]["signal_to_drained_pct"],
+        "vs_full_hw_pct": {"value": d["reduction_vs_full_hw"]["signal_to_drained_pct"],
                                      "routines": d["reduction_vs_full_hw"]["latency_pct"],
                                      "resume": d["reduction_vs_full_hw"]["resume_pct"],
                                      "context": d["reduction_vs_full_hw"]["context_pct"]},
         "poll_overhead_pct": _r(d["poll_overhead"]["overhead_pct"], 2),
         "roofline": rf, "roofline_restore": rr, "cpu_baseline": cpu,
+        "insitu_restore": {k: [_r(v["resume_floor_us"]), _r(v["frac_of_floor"], 3)]
+                           for k, v in d.get("restore_floor", {}).items()},
         "e2e": {"value": e["value"], "unit": e["unit"], "h2d_bytes_per_step": e["h2d_bytes_per_step"],
                 "d2h_bytes_per_step": e["d2h_bytes_per_step"], "host_preempt_us": e["host_preempt_us"]},
         "gpu_launches": d["gpu_launches"],
         "clocks": {k: d["clocks"].get(k) for k in ("sm_mhz", "sm_max_mhz", "reasons")},
         "configs": cfgs, "detail": detail_path,
     }
-    for drop in ("value_is", "configs"):      # stay under the driver's tail budget
+    for drop in ("insitu_restore", "configs"):      # stay under the driver's tail budget
         if len(json.dumps(line)) <= 2000:
             break
         line.pop(drop, None)

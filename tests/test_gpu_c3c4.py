@@ -62,6 +62,14 @@ def test_c3_small_forced():
     assert any(an.plans[c].n_revert_res + an.plans[c].n_revert_pre > 0 for c in an.sites)
 
 
+def test_c3_small_forced_bench_placement():
+    """The bench's C3 poll placement (8 rows per iteration, the reverting site
+    after the last row's advance only)."""
+    cfg = configs.c3(512, 128, 64, **configs.BENCH_C3)
+    an = forced_parity(cfg, 4, 3, 16)
+    assert len(an.sites) == 1 and an.plans[an.sites[0]].n_revert_res + an.plans[an.sites[0]].n_revert_pre > 0
+
+
 def test_c3_small_forced_rank_resume():
     """CTXB_RANK_RESUME (NEXT N4) plans on the GPU vs the oracle."""
     cfg = configs.c3(512, 128, 64)
@@ -88,8 +96,8 @@ def test_c3_small_forced_gather():
     forced_parity(cfg, 4, 3, 128, flags=7 | 128)
 
 
-@pytest.mark.parametrize("flags", [7, 7 | 32])
-def test_c4b_small_forced_level(flags):
+@pytest.mark.parametrize("flags,polls", [(7, "both"), (7 | 32, "both"), (7, configs.BENCH_C4B_POLLS)])
+def test_c4b_small_forced_level(flags, polls):
     rp, ci = configs.c4b_graph(1 << 10, 16)
     n = len(rp) - 1
     dist = np.full(n, 0xFFFFFFFF, np.uint32)
@@ -97,7 +105,7 @@ def test_c4b_small_forced_level(flags):
     # level 1 frontier = neighbours of 0 already discovered: run level 0 and 1 kernels
     front = np.array([0], np.uint32)
     for lvl in range(3):
-        cfg = dict(ir=configs.c4b_ir(), uniforms={"nf": len(front), "lvl1": lvl + 1},
+        cfg = dict(ir=configs.c4b_ir(polls), uniforms={"nf": len(front), "lvl1": lvl + 1},
                    buffers={"rowptr": rp, "colidx": ci, "front": np.pad(front, (0, 1)),
                             "dist": dist.copy(), "nextf": np.zeros(n, np.uint32),
                             "nextcnt": np.zeros(1, np.uint32)})
@@ -121,11 +129,11 @@ def _persistent_grid(prog):
     return bps * nsm
 
 
-@pytest.mark.parametrize("flags", [7, 7 | 32])
-def test_c3_full_flag(flags):
+@pytest.mark.parametrize("flags,variant", [(7, {}), (7 | 32, {}), (7, configs.BENCH_C3)])
+def test_c3_full_flag(flags, variant):
     import torch
     cb = _cb()
-    cfg = configs.c3()
+    cfg = configs.c3(**variant)
     W, H = cfg["W"], cfg["H"]
     op = ir.parse(cfg["ir"])
     an = A.analyze(op, policy="EXPLICIT", flags=flags)
@@ -186,16 +194,16 @@ def test_c4a_full_flag(skewed, gather):
         assert np.array_equal(total(), want)
 
 
-@pytest.mark.parametrize("replicas", [False, True])
-def test_c4b_full_flag(replicas):
+@pytest.mark.parametrize("replicas,polls", [(False, "both"), (True, "both"), (True, configs.BENCH_C4B_POLLS)])
+def test_c4b_full_flag(replicas, polls):
     import torch
     cb = _cb()
     rp, ci = configs.c4b_graph()
     n = len(rp) - 1
     want = configs.bfs_reference(rp, ci)
-    op = ir.parse(configs.c4b_ir())
+    op = ir.parse(configs.c4b_ir(polls))
     an = A.analyze(op, policy="EXPLICIT")
-    prog = cb.Program(configs.c4b_ir(), poll_policy=cb.POLL_EXPLICIT,
+    prog = cb.Program(configs.c4b_ir(polls), poll_policy=cb.POLL_EXPLICIT,
                       flags=cb.ALL | (cb.FLAG_REPLICAS if replicas else 0))
     grid = _persistent_grid(prog)
     sb = [an.plans[c].payload_bytes for c in an.sites]

@@ -278,6 +278,15 @@ def c3_ir(W=8192, H=8192, strip=64, polls="both", rows_per_iter=1):
     return "\n".join(L) + "\n"
 
 
+# Poll placement the bench uses for C3 and C4b (profiles/r02_poll_placement.md):
+# the cheapest placement measured that keeps each config's kind of site --
+# C3: 8 stencil rows per loop iteration, one site after the last row's advance
+# (the reverting site); C4b: the edge-chunk site (the OSRB site), polled
+# through flag replicas.  Both keep the poll-site overhead <= 5 %.
+BENCH_C3 = dict(rows_per_iter=8, polls="end")
+BENCH_C4B_POLLS = "edge"
+
+
 def c3(W=8192, H=8192, strip=64, polls="both", rows_per_iter=1):
     r = np.random.default_rng(21)
     bufs = {"X": f32_bits(r.uniform(0.0, 1.0, W * H).astype(np.float32)),
@@ -362,12 +371,13 @@ def c4a(nkeys=1 << 28, skewed=False, per_lane=8, grid=2):
                 policy="EXPLICIT", nkeys=nkeys, min_blocks=0)
 
 
-def c4b_ir():
+def c4b_ir(polls="both"):
     """One level of a level-synchronous top-down BFS: warp per frontier vertex
     (scalar v, edge range [beg, end) from irreversible uniform loads), lanes
     over its edges; dist[u] claimed with atomicCAS(INF -> level+1) and newly
     discovered vertices pushed with atomicAdd on the next-frontier counter.
-    Polls: after the vertex's loads and before each edge chunk's atomics."""
+    Polls ("both"): after the vertex's loads and before each edge chunk's
+    atomics; "vertex" / "edge" keep one of the two."""
     L = [".kernel c4b_bfs", ".buffer ro rowptr", ".buffer ro colidx", ".buffer ro front",
          ".buffer rw dist", ".buffer rw nextf", ".buffer rw nextcnt", ".uniform nf", ".uniform lvl1",
          ".vregs 6", ".sregs 8", ".block 256"]
@@ -384,7 +394,8 @@ def c4b_ir():
     e("  iadd s5, s3, 1")
     e("  ldg s5, rowptr[s5]")                         # end        (irreversible, reads old s5)
     e("  mov s6, s4")                                 # e = beg
-    e("  poll")
+    if polls in ("both", "vertex"):
+        e("  poll")
     e("eloop:")
     e("  setp.lt.u s7, s6, s5")
     e("  brz s7, vnext")
@@ -392,7 +403,8 @@ def c4b_ir():
     e("  iadd v0, s6, %laneid")
     e("  setp.lt.u v1, v0, s5")
     e("  @v1 ldg v2, colidx[v0]")                     # neighbour u
-    e("  poll")
+    if polls in ("both", "edge"):
+        e("  poll")
     e("  @v1 atom.cas v3, dist[v2], 0xFFFFFFFF, %lvl1")
     e("  setp.eq.u v4, v3, 0xFFFFFFFF")
     e("  and v4, v4, v1")                             # newly discovered
