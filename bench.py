@@ -475,7 +475,21 @@ def oracle_sample(steps=1, seed=0):
 MODES = (("ctxback", 0, 7), ("full_hw", 3, 7), ("live", 1, 7),
          ("cs_defer", 1, 15), ("ctxback_cs_defer", 0, 15),      # (name, mode, flags); 15 = ALL | DEFER
          ("ctxback_rank_resume", 0, 39),                        # 39 = ALL | RANK_RESUME (NEXT N4)
-         ("ctxback_gather", 0, 135), ("full_hw_gather", 3, 135))  # 135 = ALL | GATHER_RESUME
+         ("ctxback_gather", 0, 135), ("full_hw_gather", 3, 135),  # 135 = ALL | GATHER_RESUME
+         # the library gathers by default in kernels with atomics; these turn that off
+         # (debug CTXB_DEBUG_NO_AUTO_GATHER = 128; only measured for kernels with atomics)
+         ("ctxback_nogather", 0, 7, 128), ("full_hw_nogather", 3, 7, 128))
+
+
+def _modes(ir_text):
+    """(name, mode, flags, debug) of MODES that apply to the kernel."""
+    out = []
+    for m in MODES:
+        dbg = m[3] if len(m) > 3 else 0
+        if dbg & 128 and "atom." not in ir_text:
+            continue
+        out.append((m[0], m[1], m[2], dbg))
+    return out
 
 
 def poll_tuning(cb, config):
@@ -491,9 +505,9 @@ def poll_tuning(cb, config):
 
 def _progs(cb, ir_text, debug=0, min_blocks=0, extra_flags=0, load_every=1):
     return {name: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT if "poll" in ir_text else cb.POLL_EVERY_INSTR,
-                             mode=mode, flags=flags | extra_flags, debug=debug, min_blocks_per_sm=min_blocks,
+                             mode=mode, flags=flags | extra_flags, debug=debug | dbg, min_blocks_per_sm=min_blocks,
                              load_every=load_every)
-            for name, mode, flags in MODES}
+            for name, mode, flags, dbg in _modes(ir_text)}
 
 
 def _grid(progs):
@@ -593,8 +607,8 @@ def bench_c1(cb):
     cfg = configs.c1()
     names = ["in0", "in1", "rw0", "out"]
     res = {}
-    for name, mode, flags in MODES:
-        prog = cb.Program(cfg["ir"], mode=mode, flags=flags, debug=cb.DEBUG_FORCED)
+    for name, mode, flags, dbg in _modes(cfg["ir"]):
+        prog = cb.Program(cfg["ir"], mode=mode, flags=flags, debug=cb.DEBUG_FORCED | dbg)
         ctx = torch.zeros(prog.context_capacity(1), dtype=torch.uint8, device="cuda")
         dev = {n: torch.from_numpy(cfg["buffers"][n].view(np.int32).copy()).cuda() for n in names}
         ref = None

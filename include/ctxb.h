@@ -90,7 +90,8 @@ extern "C" {
                              values) keeps its greedy plan (counted in
                              ctxb_program_info_t.exact_truncated)               */
 
-#define CTXB_GATHER_RESUME 128u /* runtime: in a resume launch of a persistent grid
+#define CTXB_GATHER_RESUME 128u /* runtime (default for kernels with atomics, see
+                             CTXB_DEBUG_NO_AUTO_GATHER): in a resume launch of a persistent grid
                              (every block resident), a warp that has restored its
                              context waits until every preempted warp of the
                              launch has restored (or the flag rises again, or
@@ -184,6 +185,8 @@ extern "C" {
 #define CTXB_DEBUG_NO_COMPILE 8u /* analysis + code generation only            */
 #define CTXB_DEBUG_NO_SHARE  16u /* one preemption routine per site (no P:317
                                     sharing of identical routines)             */
+#define CTXB_DEBUG_NO_AUTO_GATHER 128u /* do not turn CTXB_GATHER_RESUME on by
+                                    default for kernels with atomics (A/B)     */
 #define CTXB_DEBUG_FENCE_STAMPS 32u /* __threadfence before the t_saved stamp, so
                                     it marks the payload as visible (slower
                                     drain; by default the kernel boundary orders
@@ -259,6 +262,9 @@ typedef struct {
   uint32_t spill_stores, spill_loads;  /* ptxas -v spill bytes of the normal kernel (0 if the
                                           log was not produced, e.g. under ncu)     */
   uint32_t spill_stores_resume, spill_loads_resume;   /* same for ctxb_resume      */
+  uint32_t gather_resume;              /* 1 if resume launches gather (CTXB_GATHER_RESUME
+                                          given, or chosen by default because the
+                                          kernel has atomics)                        */
 } ctxb_program_info_t;
 
 typedef struct {

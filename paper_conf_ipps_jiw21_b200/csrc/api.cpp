@@ -514,6 +514,14 @@ int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb
   try {
     double t0 = now_ms();
     p->prog = parse_ir(std::string(ir_text, len));
+    // Gathered resume by default for kernels with atomics:
+    // there the already-resumed warps' atomics fill the memory pipeline and
+    // the last warps' restores queue behind them (C4a: 45-130 us tails), so
+    // every resumed warp waits until all preempted warps have restored.  The
+    // policy is the framework's, so the FULL / LIVE baselines get it too.
+    bool atomics = false;
+    for (const Instr& I : p->prog.ins) atomics = atomics || I.op == Op::AtomAdd || I.op == Op::AtomCas;
+    if (atomics && !(o.debug & CTXB_DEBUG_NO_AUTO_GATHER)) p->opt.flags |= CTXB_GATHER_RESUME;
     p->an = analyze(p->prog, p->opt);
     double t1 = now_ms();
     p->src = generate_cuda(p->prog, p->an, p->opt, &p->cg);
@@ -578,6 +586,7 @@ int ctxb_program_info(const ctxb_program* p, ctxb_program_info_t* o) {
   o->spill_loads = p->spill_ld;
   o->spill_stores_resume = p->spill_st_res;
   o->spill_loads_resume = p->spill_ld_res;
+  o->gather_resume = (p->opt.flags & CTXB_GATHER_RESUME) ? 1u : 0u;
   return CTXB_OK;
 }
 

@@ -117,7 +117,7 @@ def test_runtime_options_generate_and_compile():
     (plans identical); both compile for sm_100a with NVRTC."""
     from workloads import configs
     txt = configs.c4a_ir(1 << 14)
-    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
+    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE | cb.DEBUG_NO_AUTO_GATHER)
     g = cb.Program(txt, flags=cb.ALL | cb.GATHER_RESUME | cb.SYNC_POLL, poll_policy=cb.POLL_EXPLICIT)
     assert g.info["compiled"] == 1
     assert [g.plan_text(k) for k in range(g.num_sites)] == [base.plan_text(k) for k in range(base.num_sites)]
@@ -239,3 +239,19 @@ def test_c3_unrolled_rows_parity(rows):
     for k, c in enumerate(an.sites):
         assert p.plan_text(k) == A.plan_text(op, an.plans[c])
     assert an.plans[an.sites[1]].n_revert_pre + an.plans[an.sites[1]].n_revert_res > 0
+
+
+def test_gather_resume_default_for_atomics():
+    """resume launches gather by default in kernels with
+    atomics (C4a, C4b), not otherwise (C1, C2); CTXB_DEBUG_NO_AUTO_GATHER and
+    an explicit CTXB_GATHER_RESUME override it."""
+    from workloads import configs
+    cases = [(configs.c1()["ir"], 0), (configs.c2(128, 128, 64)["ir"], 0),
+             (configs.c4a(1 << 14)["ir"], 1), (configs.c4b_ir(), 1)]
+    for txt, want in cases:
+        pol = cb.POLL_EXPLICIT if "poll" in txt else cb.POLL_EVERY_INSTR
+        assert cb.Program(txt, poll_policy=pol, debug=cb.DEBUG_NO_COMPILE).info["gather_resume"] == want
+        assert cb.Program(txt, poll_policy=pol, debug=cb.DEBUG_NO_COMPILE | cb.DEBUG_NO_AUTO_GATHER
+                          ).info["gather_resume"] == 0
+        assert cb.Program(txt, poll_policy=pol, flags=cb.ALL | cb.GATHER_RESUME,
+                          debug=cb.DEBUG_NO_COMPILE).info["gather_resume"] == 1
