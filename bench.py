@@ -330,35 +330,6 @@ def bulk_bandwidth(cb, mib, reps=5):
                 save_bytes=save_bytes, restore_bytes=rest_bytes)
 
 
-def restore_floor(cb, nvals, grid, reps=9):
-    """The cold-read floor of an in-situ restore of this size on this grid:
-    the bulk IR kernel (every warp's LIVE context = `nvals` vector values,
-    saved through the generated save stub), L2 evicted, then the resume
-    kernel's restore stub reads it back with no replay.  Device span (the
-    resume time's definition: first warp entry -> last warp restored),
-    median of `reps`.  tools/restore_micro.cu measures the same floor with a
-    hand-written read kernel (profiles/r02_restore_floor.md)."""
-    import torch
-    from workloads import configs
-    prog = cb.Program(configs.bulk_ir(nvals), poll_policy=cb.POLL_EXPLICIT, mode=cb.MODE_LIVE,
-                      debug=cb.DEBUG_FORCED, min_blocks_per_sm=2)
-    nw = grid * 8
-    out = torch.zeros(256, dtype=torch.int32, device="cuda")
-    ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
-    s = torch.cuda.Stream()
-    spans = []
-    for i in range(reps + 1):
-        run = prog.launch(grid, [out], [], ctx, s, forced=np.zeros(nw, np.uint32))
-        assert not run.wait()
-        evict_l2(s)
-        run.resume(s, forced=np.full(nw, cb.NEVER, np.uint32))
-        assert run.wait()
-        if i:
-            spans.append(run.resume_stats()["resume_us"])
-        del run
-    return float(np.median(spans))
-
-
 def poll_overhead(cb, size, grid, bufs, reps=20):
     import torch
     out = {}
@@ -1260,11 +1231,12 @@ def gpu_arm(args):
         "num_regs": pr.info["num_regs"],
     }
     # ---- cold-read floor of the in-situ restores (same bytes per warp, same grid, no replay) ----
+    # (ctxb_restore_floor: a plain read of the same layout, device-stamped like the resume time)
     floor = {}
     for k, m in (("ctxback", main), ("full_hw", base.get("full_hw"))):
         if m and m.get("context_bytes_per_tb"):
-            nv = int(round(m["context_bytes_per_tb"] / 8 / 128))
-            floor[k] = {"values_per_warp": nv, "resume_floor_us": restore_floor(cb, nv, grid),
+            bpw = int(m["context_bytes_per_tb"]) // 8
+            floor[k] = {"bytes_per_warp": bpw, "resume_floor_us": cb.ctxb_restore_floor(s, bpw, grid, 256, 9),
                         "resume_us": m["resume_us_median"]}
             floor[k]["frac_of_floor"] = floor[k]["resume_floor_us"] / max(1e-9, m["resume_us_median"])
     # ---- poll overhead, bulk roofline ----

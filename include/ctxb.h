@@ -380,6 +380,18 @@ int ctxb_query(ctxb_run* run, int* running);
  * latency as a separately measured constant).  Needs an idle GPU. */
 int ctxb_flag_propagation(void* ctrl_stream, uint32_t trials, double* median_us, double* max_us);
 
+/* Cold-read floor of a restore (measurement probe): a kernel of
+ * grid_blocks x block threads in which every warp reads its own
+ * bytes_per_warp-byte slot with the context layout's evict-first 128-bit
+ * loads and XOR-reduces it, L2 evicted before each trial (256 MiB written on
+ * `stream`); result = median over `trials` of (max over warps of "all loads
+ * returned" - min over warps of entry), %globaltimer, the definition of the
+ * resume time.  It is what a resume of that many bytes per warp on that grid
+ * costs with no dispatch, replay or register pressure.  bytes_per_warp must
+ * be a multiple of 128.  Allocates (and frees) its buffers; needs an idle GPU. */
+int ctxb_restore_floor(void* stream, uint32_t bytes_per_warp, uint32_t grid_blocks, uint32_t block,
+                       uint32_t trials, double* median_us);
+
 /* Duration of the run's last kernel launch (normal or resume), from CUDA
  * events the library records immediately before and after cuLaunchKernel on
  * the launching stream.  Valid after ctxb_wait / ctxb_preempt returned. */

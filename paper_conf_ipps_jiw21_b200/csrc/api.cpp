@@ -988,16 +988,12 @@ struct Probe {
   CUmodule mod = nullptr;
   CUfunction spin = nullptr, stamp = nullptr;
 };
-}  // namespace
 
-int ctxb_flag_propagation(void* ctrl, uint32_t trials, double* median_us, double* max_us) {
-  if (!median_us || trials == 0) return fail(CTXB_E_INVALID_ARG, "bad argument");
-  CUcontext c;
-  int rc = ensure_ctx(&c);
-  if (rc) return rc;
-  static std::mutex mu;
+std::mutex probe_mu;
+
+// The probe module of context c (compiled once with NVRTC); caller holds probe_mu.
+int probe_module(CUcontext c, Probe** out) {
   static std::map<CUcontext, Probe> probes;
-  std::lock_guard<std::mutex> g(mu);
   Probe& P = probes[c];
   Driver& d = driver();
   if (!P.mod) {
@@ -1019,6 +1015,127 @@ int ctxb_flag_propagation(void* ctrl, uint32_t trials, double* median_us, double
     CU(d.cuModuleGetFunction(&P.spin, P.mod, "ctxb_probe_spin"));
     CU(d.cuModuleGetFunction(&P.stamp, P.mod, "ctxb_probe_stamp"));
   }
+  *out = &P;
+  return CTXB_OK;
+}
+
+// Restore-floor probe: generated per slot size, like a restore stub --
+// straight-line evict-first v4 loads of every 512 B group (lane l's 16 B at
+// +16 l) and v1 loads of the 1-3 trailing 128 B rows, all issued before any
+// value is used, then an XOR reduction; stamps {entry, all loads back}.
+std::string floor_src(uint32_t slot) {
+  std::ostringstream o;
+  const uint32_t ng = slot / 512, nt = (slot % 512) / 128;
+  o << "typedef unsigned int u32; typedef unsigned long long u64;\n"
+       "static __device__ __forceinline__ u64 gt() { u64 t; asm volatile(\"mov.u64 %0, %%globaltimer;\" : \"=l\"(t)); return t; }\n"
+       "extern \"C\" __global__ void ctxb_probe_read(const unsigned char* ctx, u64* st, u32* out, u32 zero) {\n"
+       "  const u32 lane = threadIdx.x & 31u, gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;\n"
+       "  const u64 t0 = gt();\n"
+       "  const unsigned char* p = ctx + (u64)gw * " << slot << "ull;\n";
+  for (uint32_t g = 0; g < ng; g++)
+    o << "  const uint4 q" << g << " = __ldcs(reinterpret_cast<const uint4*>(p + " << g * 512 << "u) + lane);\n";
+  for (uint32_t t = 0; t < nt; t++)
+    o << "  const u32 r" << t << " = __ldcs(reinterpret_cast<const u32*>(p + " << ng * 512 + t * 128 << "u) + lane);\n";
+  o << "  u32 acc = 0u";
+  for (uint32_t g = 0; g < ng; g++) o << " ^ q" << g << ".x ^ q" << g << ".y ^ q" << g << ".z ^ q" << g << ".w";
+  for (uint32_t t = 0; t < nt; t++) o << " ^ r" << t;
+  o << ";\n  acc = __reduce_xor_sync(0xffffffffu, acc);\n"
+       "  u64 t1 = 0;\n  if ((acc & zero) == 0u) t1 = gt();\n"
+       "  if (lane == 0u) { st[(u64)gw * 2] = t0; st[(u64)gw * 2 + 1] = t1; out[gw] = acc; }\n}\n";
+  return o.str();
+}
+
+int floor_kernel(CUcontext c, uint32_t slot, CUfunction* fn) {
+  static std::map<std::pair<CUcontext, uint32_t>, CUfunction> cache;
+  auto it = cache.find({c, slot});
+  if (it != cache.end()) {
+    *fn = it->second;
+    return CTXB_OK;
+  }
+  Nvrtc& n = nvrtc();
+  if (!n.ok) return fail(CTXB_E_NVRTC, n.err);
+  std::string src = floor_src(slot);
+  void* prog = nullptr;
+  if (n.CreateProgram(&prog, src.c_str(), "floor.cu", 0, nullptr, nullptr)) return fail(CTXB_E_NVRTC, "floor probe");
+  const char* opts[] = {"--gpu-architecture=sm_100a"};
+  if (n.CompileProgram(prog, 1, opts)) {
+    n.DestroyProgram(&prog);
+    return fail(CTXB_E_NVRTC, "floor probe compile");
+  }
+  size_t cs = 0;
+  n.GetCUBINSize(prog, &cs);
+  std::vector<char> cubin(cs);
+  n.GetCUBIN(prog, cubin.data());
+  n.DestroyProgram(&prog);
+  Driver& d = driver();
+  CUmodule mod = nullptr;
+  CU(d.cuModuleLoadData(&mod, cubin.data()));
+  CU(d.cuModuleGetFunction(fn, mod, "ctxb_probe_read"));
+  cache[{c, slot}] = *fn;
+  return CTXB_OK;
+}
+}  // namespace
+
+int ctxb_restore_floor(void* stream, uint32_t bytes_per_warp, uint32_t grid_blocks, uint32_t block,
+                       uint32_t trials, double* median_us) {
+  if (!median_us || trials == 0 || grid_blocks == 0 || block == 0 || block % 32 || block > 1024 ||
+      bytes_per_warp == 0 || bytes_per_warp % 128 || bytes_per_warp > (1u << 20))
+    return fail(CTXB_E_INVALID_ARG, "bad argument");
+  CUcontext c;
+  int rc = ensure_ctx(&c);
+  if (rc) return rc;
+  std::lock_guard<std::mutex> g(probe_mu);
+  CUfunction read = nullptr;
+  if ((rc = floor_kernel(c, bytes_per_warp, &read))) return rc;
+  Driver& d = driver();
+  const uint64_t nw = (uint64_t)grid_blocks * (block / 32);
+  const size_t scratch_bytes = 256u << 20;   // > the 126 MB L2: every trial reads from HBM
+  CUdeviceptr ctx = 0, st = 0, out = 0, scr = 0;
+  CU(d.cuMemAlloc(&ctx, nw * bytes_per_warp));
+  CU(d.cuMemAlloc(&st, nw * 16));
+  CU(d.cuMemAlloc(&out, nw * 4));
+  CU(d.cuMemAlloc(&scr, scratch_bytes));
+  CUstream s = (CUstream)stream;
+  std::vector<double> v;
+  std::vector<uint64_t> h(nw * 2);
+  int err = CTXB_OK;
+  CU(d.cuMemsetD32Async(ctx, 0x5A5A5A5Au, nw * bytes_per_warp / 4, s));
+  for (uint32_t t = 0; t <= trials && !err; t++) {
+    uint32_t zero = 0;
+    void* a[] = {&ctx, &st, &out, &zero};
+    if (d.cuMemsetD32Async(scr, t, scratch_bytes / 4, s) != CUDA_SUCCESS ||
+        d.cuLaunchKernel(read, grid_blocks, 1, 1, block, 1, 1, 0, s, a, nullptr) != CUDA_SUCCESS ||
+        d.cuStreamSynchronize(s) != CUDA_SUCCESS || d.cuMemcpyDtoH(h.data(), st, nw * 16) != CUDA_SUCCESS) {
+      err = fail(CTXB_E_CUDA, "restore floor probe failed");
+      break;
+    }
+    uint64_t a0 = UINT64_MAX, b0 = 0;
+    for (uint64_t w = 0; w < nw; w++) {
+      a0 = std::min(a0, h[w * 2]);
+      b0 = std::max(b0, h[w * 2 + 1]);
+    }
+    if (t) v.push_back((double)(b0 - a0) * 1e-3);   // the first trial is a warm-up
+  }
+  d.cuMemFree(ctx);
+  d.cuMemFree(st);
+  d.cuMemFree(out);
+  d.cuMemFree(scr);
+  if (err) return err;
+  std::sort(v.begin(), v.end());
+  *median_us = v[v.size() / 2];
+  return CTXB_OK;
+}
+
+int ctxb_flag_propagation(void* ctrl, uint32_t trials, double* median_us, double* max_us) {
+  if (!median_us || trials == 0) return fail(CTXB_E_INVALID_ARG, "bad argument");
+  CUcontext c;
+  int rc = ensure_ctx(&c);
+  if (rc) return rc;
+  std::lock_guard<std::mutex> g(probe_mu);
+  Probe* PP = nullptr;
+  if ((rc = probe_module(c, &PP))) return rc;
+  Probe& P = *PP;
+  Driver& d = driver();
   CUdeviceptr flag = 0, out = 0;
   CU(d.cuMemAlloc(&flag, 256));
   CU(d.cuMemAlloc(&out, 64));

@@ -19,7 +19,7 @@ __all__ = [
     "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS", "DEBUG_NO_AUTO_GATHER",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "E_TIMEOUT", "EXPORTED_SYMBOLS",
     "ctxb_analyze", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait", "ctxb_context_bytes",
-    "ctxb_flag_propagation",
+    "ctxb_flag_propagation", "ctxb_restore_floor",
     "Program", "Run",
 ]
 
@@ -41,7 +41,7 @@ EXPORTED_SYMBOLS = [
     "ctxb_num_sites", "ctxb_site_info", "ctxb_backups", "ctxb_site_plan_text", "ctxb_generated_source",
     "ctxb_occupancy", "ctxb_context_capacity", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait",
     "ctxb_query", "ctxb_flag_propagation", "ctxb_launch_ms", "ctxb_resume_stats_get", "ctxb_context_bytes", "ctxb_read_headers", "ctxb_read_stamps",
-    "ctxb_run_destroy", "ctxb_preempt_async", "ctxb_program_cubin",
+    "ctxb_run_destroy", "ctxb_preempt_async", "ctxb_program_cubin", "ctxb_restore_floor",
 ]
 
 
@@ -119,6 +119,7 @@ def _load():
         "ctxb_run_destroy": (I, [P]),
         "ctxb_preempt_async": (I, [P, P]),
         "ctxb_program_cubin": (I, [P, P, SZ, C.POINTER(SZ)]),
+        "ctxb_restore_floor": (I, [P, U32, U32, U32, U32, C.POINTER(C.c_double)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -193,6 +194,16 @@ def ctxb_flag_propagation(ctrl_stream, trials=20):
     m, x = C.c_double(), C.c_double()
     _chk(lib.ctxb_flag_propagation(_stream(ctrl_stream), trials, C.byref(m), C.byref(x)))
     return m.value, x.value
+
+
+def ctxb_restore_floor(stream, bytes_per_warp, grid, block=256, trials=9):
+    """Cold-read floor (us) of restoring bytes_per_warp (rounded up to 128) per
+    warp on a grid x block launch: device span of a plain read of the same
+    layout, L2 evicted before each trial."""
+    m = C.c_double()
+    b = (int(bytes_per_warp) + 127) // 128 * 128
+    _chk(lib.ctxb_restore_floor(_stream(stream), b, grid, block, trials, C.byref(m)))
+    return m.value
 
 
 class Program:

@@ -189,3 +189,15 @@ def test_ctrl_stream_checks():
     if st["warps_preempted"]:
         run.resume(s)
     assert run.wait()
+
+
+def test_restore_floor_probe():
+    """ctxb_restore_floor: device span of a plain cold read of the context
+    layout; positive and growing with the bytes per warp."""
+    import torch
+    cb = _cb()
+    s = torch.cuda.Stream()
+    f = [cb.ctxb_restore_floor(s, b, 296, 256, 3) for b in (2048, 8832, 16384)]
+    assert 0 < f[0] < f[1] < f[2], f
+    m = __import__("ctypes").c_double()
+    assert cb.lib.ctxb_restore_floor(None, 100, 296, 256, 3, __import__("ctypes").byref(m)) == -1   # not a multiple of 128
