@@ -184,9 +184,12 @@ extern "C" {
                                     the kernel cannot be preempted)            */
 #define CTXB_DEBUG_NO_COMPILE 8u /* analysis + code generation only            */
 #define CTXB_DEBUG_NO_SHARE  16u /* one preemption routine per site (no P:317
-                                    sharing of identical routines)             */
+                                    sharing at all)                            */
 #define CTXB_DEBUG_NO_AUTO_GATHER 128u /* do not turn CTXB_GATHER_RESUME on by
                                     default for kernels with atomics (A/B)     */
+#define CTXB_DEBUG_NO_FP_SHARE 256u /* keep only the exact sharing of byte-identical
+                                    preemption routines: no per-flashback-point
+                                    routine with entry offsets (A/B)    */
 #define CTXB_DEBUG_FENCE_STAMPS 32u /* __threadfence before the t_saved stamp, so
                                     it marks the payload as visible (slower
                                     drain; by default the kernel boundary orders
@@ -265,6 +268,9 @@ typedef struct {
   uint32_t gather_resume;              /* 1 if resume launches gather (CTXB_GATHER_RESUME
                                           given, or chosen by default because the
                                           kernel has atomics)                        */
+  uint32_t n_fp_shared;                /* sites whose preemption routine is their
+                                          flashback-point's shared routine, entered at
+                                          an offset past the later sites' reverts */
 } ctxb_program_info_t;
 
 typedef struct {

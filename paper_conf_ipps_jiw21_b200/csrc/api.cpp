@@ -587,6 +587,7 @@ int ctxb_program_info(const ctxb_program* p, ctxb_program_info_t* o) {
   o->spill_stores_resume = p->spill_st_res;
   o->spill_loads_resume = p->spill_ld_res;
   o->gather_resume = (p->opt.flags & CTXB_GATHER_RESUME) ? 1u : 0u;
+  o->n_fp_shared = p->cg.n_fp_shared;
   return CTXB_OK;
 }
 

@@ -176,6 +176,7 @@ struct CodegenInfo {
   uint32_t max_payload = 0;
   uint32_t resume_maxnreg = 0;    // in: register cap of the resume kernel (0 = none)
   uint32_t n_save_stubs = 0;      // out: distinct preemption-routine bodies (P:317 sharing)
+  uint32_t n_fp_shared = 0;       // out: sites entering a flashback-point routine at an offset
 };
 std::string generate_cuda(const Program& prog, const Analysis& an, const Options& opt,
                           CodegenInfo* info);

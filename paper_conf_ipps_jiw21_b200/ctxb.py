@@ -16,7 +16,7 @@ __all__ = [
     "LIB_PATH", "CtxbError", "lib",
     "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "GATHER_RESUME", "SYNC_POLL", "HOST_SIGNAL", "ARMED_SIGNAL", "OSRB_SMEM", "OSRB_LANES", "FLAG_REPLICAS", "DRAIN_NOTICE", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
-    "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS", "DEBUG_NO_AUTO_GATHER",
+    "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS", "DEBUG_NO_AUTO_GATHER", "DEBUG_NO_FP_SHARE",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "E_TIMEOUT", "EXPORTED_SYMBOLS",
     "ctxb_analyze", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait", "ctxb_context_bytes",
     "ctxb_flag_propagation", "ctxb_restore_floor",
@@ -31,7 +31,7 @@ ARMED_SIGNAL, OSRB_SMEM, OSRB_LANES, FLAG_REPLICAS, DRAIN_NOTICE = 1024, 2048, 4
 MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
 DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1, 2, 4, 8, 16
-DEBUG_FENCE_STAMPS, DEBUG_NO_AUTO_GATHER = 32, 128
+DEBUG_FENCE_STAMPS, DEBUG_NO_AUTO_GATHER, DEBUG_NO_FP_SHARE = 32, 128, 256
 STATE_NONE, STATE_PREEMPTED, STATE_DONE = 0, 1, 2
 NEVER = 0xFFFFFFFF
 E_TIMEOUT = -8   # ctxb_preempt gave up waiting (env CTXB_PREEMPT_TIMEOUT_US)
@@ -72,7 +72,7 @@ class _ProgInfo(C.Structure):
                                           "exact_improved", "exact_fallback")] + \
                [("analyze_ms", C.c_double), ("codegen_ms", C.c_double), ("compile_ms", C.c_double)] + \
                [(n, C.c_uint32) for n in ("spill_stores", "spill_loads", "spill_stores_resume", "spill_loads_resume",
-                                          "gather_resume")]
+                                          "gather_resume", "n_fp_shared")]
 
 
 class _PreStats(C.Structure):
