@@ -296,7 +296,7 @@ def bulk_bandwidth(cb, mib, reps=5):
     import torch
     from workloads import configs
     prog = cb.Program(configs.bulk_ir(64), poll_policy=cb.POLL_EXPLICIT, mode=cb.MODE_LIVE,
-                      debug=cb.DEBUG_FORCED)
+                      debug=cb.DEBUG_FORCED, min_blocks_per_sm=configs.BULK_MIN_BLOCKS)
     per_warp = 64 * 128
     nw = (mib << 20) // per_warp
     grid = nw // 8

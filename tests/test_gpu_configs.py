@@ -116,7 +116,7 @@ def test_bulk_save_restore_roundtrip():
     import torch
     cb = _cb()
     prog = cb.Program(configs.bulk_ir(64), poll_policy=cb.POLL_EXPLICIT, mode=cb.MODE_LIVE,
-                      debug=cb.DEBUG_FORCED)
+                      debug=cb.DEBUG_FORCED, min_blocks_per_sm=configs.BULK_MIN_BLOCKS)
     grid = 2048
     nw = grid * 8
     out = torch.zeros(256, dtype=torch.int32, device="cuda")

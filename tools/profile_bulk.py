@@ -12,7 +12,7 @@ import paper_conf_ipps_jiw21_b200 as cb  # noqa: E402
 from workloads import configs  # noqa: E402
 
 mib = int(sys.argv[1]) if len(sys.argv) > 1 else 1024
-prog = cb.Program(configs.bulk_ir(64), poll_policy=cb.POLL_EXPLICIT, mode=cb.MODE_LIVE, debug=cb.DEBUG_FORCED)
+prog = cb.Program(configs.bulk_ir(64), poll_policy=cb.POLL_EXPLICIT, mode=cb.MODE_LIVE, debug=cb.DEBUG_FORCED, min_blocks_per_sm=configs.BULK_MIN_BLOCKS)
 nw = (mib << 20) // (64 * 128)
 grid = nw // 8
 nw = grid * 8

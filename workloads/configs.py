@@ -180,6 +180,13 @@ def c2(M=4096, N=4096, K=4096, grid=None, polls="iter"):
                 M=M, N=N, K=K)
 
 
+# Resident blocks per SM for the bulk kernels: caps both generated kernels at
+# the same register budget (77 / 76 registers, 24 warps per SM) so neither
+# spills (the compiler's own choice rematerialises the values in the save
+# kernel and spills 56 B in the resume kernel, profiles/r02_sass.md).
+BULK_MIN_BLOCKS = 3
+
+
 def bulk_ir(nvals=64, block=256):
     """Bulk save/restore microbench (SURVEY §8(d) '>=70 % gate'): every thread
     builds `nvals` live vector values from its thread id, then polls once; in
