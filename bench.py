@@ -59,9 +59,11 @@ def parse():
                          "stream, standing in for the LS job, so the context is read back from HBM)")
     ap.add_argument("--detail", default=os.path.join(ROOT, "gpurun_out", "bench_detail.json"),
                     help="side file for the full result (per-config, C5, baselines); stdout gets a compact line")
-    ap.add_argument("--signal", default="armed", choices=["armed", "memop"],
-                    help="C2 preemption signal of the headline modes: armed = CTXB_ARMED_SIGNAL (pre-enqueued "
-                         "behind a host gate, DESIGN.md 8j); memop = cuStreamWriteValue32 on the control stream")
+    ap.add_argument("--signal", default="watcher", choices=["watcher", "armed", "memop"],
+                    help="preemption signal of the headline modes: watcher = CTXB_WATCHER | CTXB_DRAIN_NOTICE (a "
+                         "co-resident warp relays a host store; the last warp's exit is noticed in host memory, "
+                         "DESIGN.md 8n); armed = CTXB_ARMED_SIGNAL (pre-enqueued memop behind a host gate, 8j); "
+                         "memop = cuStreamWriteValue32 on the control stream")
     return ap.parse_args()
 
 
@@ -171,7 +173,12 @@ class Clocks:
 
 # ---- the GPU arm --------------------------------------------------------------
 
-SIGNAL_FLAGS = 0   # set by gpu_arm from --signal: cb.ARMED_SIGNAL or 0
+SIGNAL_FLAGS = 0   # set by gpu_arm from --signal (signal_paths)
+
+
+def signal_paths(cb):
+    """--signal name -> program flags of that preemption-signal path."""
+    return {"watcher": cb.WATCHER | cb.DRAIN_NOTICE, "armed": cb.ARMED_SIGNAL, "memop": 0}
 C3_ROWS = 8        # C3 stencil rows per loop iteration, one (reverting) poll site per iteration (configs.BENCH_C3)
 
 
@@ -482,11 +489,8 @@ def _progs(cb, ir_text, debug=0, min_blocks=0, extra_flags=0, load_every=1):
 
 
 def _grid(progs):
-    bps, nsm = None, None
-    for p in progs.values():
-        b, nsm = p.occupancy()
-        bps = b if bps is None else min(bps, b)
-    return bps * nsm
+    """One persistent grid for every mode of a config (ctxb_persistent_grid)."""
+    return min(p.persistent_grid() for p in progs.values())
 
 
 def _static(prog, nwarps):
@@ -539,21 +543,23 @@ def _flag_trials(progs, grid, make_bufs, uniforms, check, fracs, T_s):
 def _poll_overhead(cb, ir_text, grid, make_bufs, uniforms=(), extra_flags=0, min_blocks=0, reps=9, load_every=1):
     """Poll-site (+OSRB copy) overhead, the paper's Fig. 10 quantity: the
     uninterrupted CTXBack kernel vs the same generated kernel with the poll
-    sites compiled out (CTXB_DEBUG_NO_POLLS), medians of `reps` launches."""
-    out = {}
+    sites compiled out (CTXB_DEBUG_NO_POLLS), medians of `reps` launches of
+    each, interleaved (so clock or thermal drift hits both alike)."""
+    import torch
+    progs, ctxs, ts = {}, {}, {}
     for name, dbg in (("polls_ms", 0), ("no_polls_ms", cb.DEBUG_NO_POLLS)):
-        prog = cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | extra_flags, debug=dbg,
-                          min_blocks_per_sm=min_blocks, load_every=load_every)
-        import torch
-        ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
-        ts = []
-        for i in range(reps + 1):
-            run = prog.launch(grid, make_bufs(), list(uniforms), ctx)
+        progs[name] = cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | extra_flags, debug=dbg,
+                                 min_blocks_per_sm=min_blocks, load_every=load_every)
+        ctxs[name] = torch.empty(progs[name].context_capacity(grid), dtype=torch.uint8, device="cuda")
+        ts[name] = []
+    for i in range(reps + 1):
+        for name, prog in progs.items():
+            run = prog.launch(grid, make_bufs(), list(uniforms), ctxs[name])
             run.wait()
             if i:
-                ts.append(run.launch_ms())
+                ts[name].append(run.launch_ms())
             del run
-        out[name] = float(np.median(ts))
+    out = {name: float(np.median(v)) for name, v in ts.items()}
     out["overhead_pct"] = 100.0 * (out["polls_ms"] / out["no_polls_ms"] - 1.0)
     return out
 
@@ -643,7 +649,7 @@ def bench_c2s(cb, trials, seed):
     res = _flag_trials(progs, grid, make, [], lambda b_: bool(torch.equal(b_[2], ref)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
     res["static"]["smem_bytes_per_tb"] = 4 * 2048
-    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], grid, make, min_blocks=2)
+    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], progs["ctxback"].persistent_grid(), make, min_blocks=2)
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
@@ -677,7 +683,8 @@ def bench_c3(cb, trials, seed):
     fr = np.random.default_rng(seed + 2).uniform(0.05, 0.95, trials)
     res = _flag_trials(progs, grid, make, [], lambda b: bool(torch.equal(b[1], ref)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
-    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], grid, make, **poll_tuning(cb, "c3"))
+    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], progs["ctxback"].persistent_grid(), make,
+                                          **poll_tuning(cb, "c3"))
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
@@ -717,7 +724,10 @@ def bench_c4a(cb, trials, seed):
     fr = np.random.default_rng(seed + 3).uniform(0.05, 0.95, trials)
     res = _flag_trials(progs, grid, make, [], lambda b: bool(torch.equal(hsum(b[2]), want)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
-    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], grid, make, **poll_tuning(cb, "c4a"))   # incl. the OSRB copy
+    g_own = progs["ctxback"].persistent_grid()   # the CTXBack kernel's own persistent grid
+    if g_own > grid:
+        dH = torch.zeros(256 * g_own, dtype=torch.int32, device="cuda")
+    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], g_own, make, **poll_tuning(cb, "c4a"))   # incl. the OSRB copy
     osrb_off = cb.Program(cfg["ir"], flags=cb.RELAXED | cb.REVERT, poll_policy=cb.POLL_EXPLICIT,
                           debug=cb.DEBUG_NO_COMPILE)
     res["static"]["ctxback_osrb_off_bytes_per_tb_per_site"] = [
@@ -793,7 +803,7 @@ def bench_c4b(cb, trials, seed):
         res[name] = summarize(recs)
     res["static"] = _static(progs["ctxback"], 8)
 
-    def bfs_ms(prog):
+    def bfs_ms(prog, grid=grid):
         """All levels uninterrupted: summed kernel time."""
         ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
         d_dist.fill_(-1)
@@ -810,12 +820,17 @@ def bench_c4b(cb, trials, seed):
             nf = int(cnt.item())
             lvl += 1
         return tot
-    ov = {}
-    for key, dbg in (("polls_ms", 0), ("no_polls_ms", cb.DEBUG_NO_POLLS)):
-        pr = cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, debug=dbg,
-                        flags=cb.ALL | poll_tuning(cb, "c4b").get("extra_flags", 0))
-        bfs_ms(pr)
-        ov[key] = float(np.median([bfs_ms(pr) for _ in range(5)]))
+    prs = {key: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, debug=dbg,
+                           flags=cb.ALL | poll_tuning(cb, "c4b").get("extra_flags", 0))
+           for key, dbg in (("polls_ms", 0), ("no_polls_ms", cb.DEBUG_NO_POLLS))}
+    tv = {key: [] for key in prs}
+    g_own = prs["polls_ms"].persistent_grid()   # the CTXBack kernel's own persistent grid
+    for i in range(10):                       # interleaved: drift hits both alike
+        for key, pr in prs.items():
+            t_ = bfs_ms(pr, g_own)
+            if i:
+                tv[key].append(t_)
+    ov = {key: float(np.median(v)) for key, v in tv.items()}
     ov["overhead_pct"] = 100.0 * (ov["polls_ms"] / ov["no_polls_ms"] - 1.0)
     res["poll_overhead"] = ov
     res["reduction_vs_full_hw"] = _reduction(res)
@@ -913,8 +928,7 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
             progs[k] = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, mode=mode_id[mode], min_blocks_per_sm=mb,
                                   flags=cb.ALL | tune.get("extra_flags", 0) | (SIGNAL_FLAGS if mode != "none" else 0),
                                   load_every=tune.get("load_every", 1))
-            b_, nsm = progs[k].occupancy()
-            grids[k] = b_ * nsm
+            grids[k] = progs[k].persistent_grid()
             ctxs[k] = torch.empty(progs[k].context_capacity(grids[k]), dtype=torch.uint8, device="cuda")
         dev["H"] = torch.zeros(256 * grids["c4a"], dtype=torch.int32, device="cuda")
 
@@ -1156,7 +1170,7 @@ def gpu_arm(args):
     import paper_conf_ipps_jiw21_b200 as cb
     from workloads import configs
     global SIGNAL_FLAGS, WARM_RESUME
-    SIGNAL_FLAGS = cb.ARMED_SIGNAL if args.signal == "armed" else 0
+    SIGNAL_FLAGS = signal_paths(cb)[args.signal]
     WARM_RESUME = args.warm_resume
     ws, rank, local = dist_setup(args)
     torch.cuda.set_device(local)
@@ -1173,17 +1187,15 @@ def gpu_arm(args):
         # CTXB_GATHER_RESUME: resumed warps wait until every preempted warp has restored
         progs["ctxback_gather"] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | cb.GATHER_RESUME | SIGNAL_FLAGS)
         progs["full_hw_gather"] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | cb.GATHER_RESUME | SIGNAL_FLAGS)
-        # the other signal path next to the headline's
-        other, oname = (0, "memop") if SIGNAL_FLAGS else (cb.ARMED_SIGNAL, "armed")
-        progs["ctxback_" + oname] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | other)
-        progs["full_hw_" + oname] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | other)
-        # CTXB_DRAIN_NOTICE: the host learns "drained" from a host-memory word the last warp writes
-        progs["ctxback_notice"] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | SIGNAL_FLAGS | cb.DRAIN_NOTICE)
-        progs["full_hw_notice"] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | SIGNAL_FLAGS | cb.DRAIN_NOTICE)
-    bps, nsm = progs["ctxback"].occupancy()
-    for p in progs.values():
-        bps = min(bps, p.occupancy()[0])
-    grid = bps * nsm
+        # the other signal paths next to the headline's
+        for oname, other in signal_paths(cb).items():
+            if oname != args.signal:
+                progs["ctxback_" + oname] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | other)
+                progs["full_hw_" + oname] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | other)
+    # one persistent grid for every mode (room for the watcher warp where a mode uses it)
+    grid = min(p.persistent_grid() for p in progs.values())
+    nsm = progs["ctxback"].occupancy()[1]
+    bps = -(-grid // nsm)
     dA = torch.from_numpy(cfg["buffers"]["A"].view(np.int32)).cuda()
     dB = torch.from_numpy(cfg["buffers"]["B"].view(np.int32)).cuda()
     dC = torch.zeros(M * N, dtype=torch.int32, device="cuda")
@@ -1214,8 +1226,8 @@ def gpu_arm(args):
     main = summarize(recs)
     # ---- baselines in the same framework (same fracs) ----
     base = {}
-    for k in ("full_hw", "full_ir", "live", "ctxback_gather", "full_hw_gather", "ctxback_armed", "full_hw_armed",
-              "ctxback_memop", "full_hw_memop", "ctxback_notice", "full_hw_notice"):
+    for k in ("full_hw", "full_ir", "live", "ctxback_gather", "full_hw_gather", "ctxback_watcher", "full_hw_watcher",
+              "ctxback_armed", "full_hw_armed", "ctxback_memop", "full_hw_memop"):
         if k in progs:
             preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_w[:1], ws)
             r = preempt_steps(cb, progs[k], grid, (dA, dB, dC), ctxs[k], s, ctrl, ref, t_unint_ms / 1e3, fr_t, ws)
@@ -1288,7 +1300,7 @@ def gpu_arm(args):
     e2e_val = float(np.median([x["step_us"] for x in e2e]))
     e2e_host = float(np.median([x["host_us"] for x in e2e if x["pre"]] or [0.0]))
     # ---- max over ranks ----
-    value = allmax(ws, main.get("signal_to_drained_us_median") or main["latency_us_median"])
+    value = allmax(ws, main["host_latency_us_median"])
     ms_per_step = allmax(ws, float(np.mean([r["step_ms"] for r in recs])))
     c5_total = None
     if "c5" in extra_cfg:
@@ -1332,10 +1344,10 @@ def gpu_arm(args):
                                  "for the LS job), so every resume reads its context from HBM"),
                    "parallelism": f"replicas x{ws}"},
         "resume_us": round(main["resume_us_median"], 3),
-        "value_definition": ("median over steps of signal -> all blocks drained: CUDA event right before the flag "
-                             "write on the signal's stream (--signal armed: libctxb's signal stream, the event runs "
-                             "once the host gate opened; memop: the caller's control stream) -> libctxb's event "
-                             "after the victim kernel (every warp saved or finished, kernel exited)"),
+        "value_definition": ("median over steps of the host-observed preemption latency: ctxb_preempt entry -> "
+                             "the host knows every warp of the victim saved its context or finished (host clock, "
+                             f"inside libctxb; signal path '{args.signal}'); signal_to_drained_us_median (CUDA events, "
+                             "memop paths only) is reported beside it"),
         "preemption_routines_us": round(main["latency_us_median"], 3),
         "preemption_routines_definition": "max t_saved - min t_flag_seen over preempted warps (%globaltimer)",
         "flag_propagation_us": {"median": round(prop_med, 3), "max": round(prop_max, 3),
@@ -1345,6 +1357,9 @@ def gpu_arm(args):
         "context_bytes_per_tb": main.get("context_bytes_per_tb"),
         "ctxback": main, "baselines": base, "static_context": static,
         "reduction_vs_full_hw": {
+            "host_latency_pct": (round(100 * (1 - main["host_latency_us_median"] /
+                                              base["full_hw"]["host_latency_us_median"]), 2)
+                                 if "full_hw" in base and base["full_hw"].get("host_latency_us_median") else None),
             "signal_to_drained_pct": (round(100 * (1 - main["signal_to_drained_us_median"] /
                                                    base["full_hw"]["signal_to_drained_us_median"]), 2)
                                       if "full_hw" in base and base["full_hw"].get("signal_to_drained_us_median")
@@ -1358,7 +1373,10 @@ def gpu_arm(args):
                             main.get("context_bytes_per_tb") else None)},
         "signal": args.signal,
         "other_signal_reduction": {k: _reduction(base, "ctxback_" + k, "full_hw_" + k)
-                                   for k in ("armed", "memop", "notice") if "ctxback_" + k in base},
+                                   for k in ("watcher", "armed", "memop") if "ctxback_" + k in base},
+        "other_signal_host_latency_us": {k: [base.get("ctxback_" + k, {}).get("host_latency_us_median"),
+                                             base.get("full_hw_" + k, {}).get("host_latency_us_median")]
+                                         for k in ("watcher", "armed", "memop") if "ctxback_" + k in base},
         "poll_overhead": ovh, "bulk": bulk, "configs": extra_cfg, "restore_floor": floor,
         "roofline": rf, "roofline_restore": rr,
         # the victim whose polls are measured: C2's FFMA SGEMM against the FP32 ALU peak
@@ -1426,9 +1444,10 @@ def compact_line(d, detail_path):
                    "l2": "inputs > L2; resume L2-cold" if "cold" in d["config"]["resume_l2"] else "inputs > L2; resume warm"},
         "routines_us": _r(m["latency_us_median"], 3), "resume_us": _r(m["resume_us_median"], 3),
         "context_bytes_per_tb": m.get("context_bytes_per_tb"),
-        "full_hw": {"value": _r(fh.get("signal_to_drained_us_median"), 3), "routines_us": _r(fh.get("latency_us_median"), 3),
+        "signal": d["signal"],
+        "full_hw": {"value": _r(fh.get("host_latency_us_median"), 3), "routines_us": _r(fh.get("latency_us_median"), 3),
                     "resume_us": _r(fh.get("resume_us_median"), 3), "context_bytes_per_tb": fh.get("context_bytes_per_tb")},
-        "vs_full_hw_pct": {"value": d["reduction_vs_full_hw"]["signal_to_drained_pct"],
+        "vs_full_hw_pct": {"value": d["reduction_vs_full_hw"]["host_latency_pct"],
                                      "routines": d["reduction_vs_full_hw"]["latency_pct"],
                                      "resume": d["reduction_vs_full_hw"]["resume_pct"],
                                      "context": d["reduction_vs_full_hw"]["context_pct"]},
@@ -1473,6 +1492,9 @@ def reference_arm(args):
 
 
 def main():
+    if os.environ.get("BENCH_HANG_DUMP_S"):      # debugging aid: dump every thread's stack, then exit
+        import faulthandler
+        faulthandler.dump_traceback_later(float(os.environ["BENCH_HANG_DUMP_S"]), exit=True)
     args = parse()
     if args.impl == "reference":
         line = reference_arm(args)

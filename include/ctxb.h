@@ -163,6 +163,23 @@ extern "C" {
                              (the sysmem write is flushed at kernel end) comes
                              ~2 µs later                      */
 
+#define CTXB_WATCHER 32768u /* runtime: every launch (and resume) first starts a
+                             one-warp watcher kernel on a library-owned
+                             greatest-priority stream; the launch waits (stream
+                             memory op) until it runs, so it is co-resident with
+                             the victim (ctxb_persistent_grid leaves room for
+                             it).  ctxb_preempt stores the launch's sequence
+                             number to a word in mapped pinned host memory; the
+                             watcher polls that word with system-scope loads and
+                             raises the device flag (+ replicas), bypassing the
+                             ~7 us stream memory op, which stays as the fallback
+                             on ctrl_stream (env CTXB_HOST_SIGNAL_ONLY=1 drops
+                             it: tests).  A launch that ends unpreempted
+                             releases its watcher when collected.
+                             signal_to_drained_us is 0 (the host store is not
+                             stream-ordered): use host_us.  Exclusive with
+                             CTXB_ARMED_SIGNAL (_INVALID_ARG)                  */
+
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */
 #define CTXB_MODE_FULL    2u /* save every declared IR register (FULL_IR)        */
@@ -327,6 +344,12 @@ int ctxb_program_cubin(const ctxb_program* prog, void* buf, size_t cap, size_t* 
  * persistent grid is blocks_per_sm * num_sms ("persistent thread").
  * Needs a GPU (_CUDA otherwise). */
 int ctxb_occupancy(ctxb_program* prog, uint32_t* blocks_per_sm, uint32_t* num_sms);
+
+/* The largest grid whose blocks are all resident at once ("persistent
+ * thread"): blocks_per_sm * num_sms, one block fewer when the program uses
+ * CTXB_WATCHER and the watcher warp does not fit next to blocks_per_sm
+ * blocks on an SM.  Needs a GPU. */
+int ctxb_persistent_grid(ctxb_program* prog, uint32_t* grid);
 
 /* Bytes of device memory a context buffer for `grid_blocks` blocks needs:
  * 16 B header per warp + per-warp payload slots. */

@@ -124,6 +124,8 @@ struct ctxb_run {
   CUstream arm = nullptr;   // CTXB_ARMED_SIGNAL: stream holding the pre-enqueued signal
   uint32_t gate_seq = 0;    //   gate value that releases the armed signal of the current launch
   bool armed = false;       //   an armed signal is pending on `arm`
+  bool watching = false;    // CTXB_WATCHER: the current launch's watcher warp waits for the host word
+  CUdeviceptr stamps_watch = 0;   //   where the watcher stamps when it raised the flag (stamps + 32 n_warps)
   uint32_t epoch = 0;
   uint32_t rb_target = 0;   // CTXB_GATHER_RESUME: blocks with preempted warps the resume launch waits for
   int state = RUN_RUNNING;
@@ -138,6 +140,12 @@ struct ctxb_run {
   // CTXB_ARMED_SIGNAL: release a pending armed signal of a launch that was not
   // preempted and clear the flag it raises (off the preemption path).
   void disarm() {
+    if (watching) {   // CTXB_WATCHER: the launch ended unpreempted -> the watcher exits
+      watching = false;
+      *(static_cast<volatile uint32_t*>(hflag) + 8) = gate_seq | 0x80000000u;
+      std::atomic_thread_fence(std::memory_order_seq_cst);
+      driver().cuStreamSynchronize(arm);
+    }
     if (!armed) return;
     armed = false;
     Driver& d = driver();
@@ -406,6 +414,152 @@ int write_signal(ctxb_run* r, CUstream s) {
   return CTXB_OK;
 }
 
+const char* kProbeSrc = R"CUDA(
+typedef unsigned int u32; typedef unsigned long long u64;
+static __device__ __forceinline__ u64 gt() { u64 t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); return t; }
+static __device__ __forceinline__ u32 ldcv(const u32* p) { u32 v; asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p)); return v; }
+extern "C" __global__ void ctxb_probe_spin(const u32* flag, u64* out) {
+  u64 t0 = gt();
+  while (ldcv(flag) == 0u) { if (gt() - t0 > 20000000ull) break; }   // 20 ms timeout
+  if (threadIdx.x == 0) out[1] = gt();
+}
+extern "C" __global__ void ctxb_probe_stamp(u64* out) { if (threadIdx.x == 0) out[0] = gt(); }
+// CTXB_WATCHER: one warp, co-resident with the victim, relays a host store to
+// the device flag.  It marks itself started (the victim's launch waits for
+// that, so the watcher always has its slot), then polls the host word in
+// mapped pinned memory with system-scope loads: seq raises the launch's signal
+// value in the master flag and every replica; seq | 0x80000000 (the launch
+// ended unpreempted) makes it exit.
+extern "C" __global__ void ctxb_watcher(const u32* hw, u32 seq, u32* flag, unsigned long long rep_off, u32 sig,
+                                        u32* started, u64* stamp) {
+  const u32 lane = threadIdx.x;
+  if (lane == 0) asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(started), "r"(seq) : "memory");
+  u32 v;
+  do { asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(hw) : "memory"); }
+  while (v != seq && v != (seq | 0x80000000u));
+  if (v != seq) return;
+  for (u32 k = lane; k <= 64u; k += 32u) {
+    u32* a = k == 0u ? flag : flag + (rep_off + (u64)(k - 1u) * 4096u) / 4u;
+    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(a), "r"(sig) : "memory");
+  }
+  if (lane == 0) *stamp = gt();
+}
+)CUDA";
+
+struct Probe {
+  CUmodule mod = nullptr;
+  CUfunction spin = nullptr, stamp = nullptr, watch = nullptr;
+};
+
+std::mutex probe_mu;
+
+// The probe module of context c (compiled once with NVRTC); caller holds probe_mu.
+int probe_module(CUcontext c, Probe** out) {
+  static std::map<CUcontext, Probe> probes;
+  Probe& P = probes[c];
+  Driver& d = driver();
+  if (!P.mod) {
+    Nvrtc& n = nvrtc();
+    if (!n.ok) return fail(CTXB_E_NVRTC, n.err);
+    void* prog = nullptr;
+    if (n.CreateProgram(&prog, kProbeSrc, "probe.cu", 0, nullptr, nullptr)) return fail(CTXB_E_NVRTC, "probe");
+    const char* opts[] = {"--gpu-architecture=sm_100a"};
+    if (n.CompileProgram(prog, 1, opts)) {
+      n.DestroyProgram(&prog);
+      return fail(CTXB_E_NVRTC, "probe compile");
+    }
+    size_t cs = 0;
+    n.GetCUBINSize(prog, &cs);
+    std::vector<char> cubin(cs);
+    n.GetCUBIN(prog, cubin.data());
+    n.DestroyProgram(&prog);
+    CU(d.cuModuleLoadData(&P.mod, cubin.data()));
+    CU(d.cuModuleGetFunction(&P.spin, P.mod, "ctxb_probe_spin"));
+    CU(d.cuModuleGetFunction(&P.stamp, P.mod, "ctxb_probe_stamp"));
+    CU(d.cuModuleGetFunction(&P.watch, P.mod, "ctxb_watcher"));
+  }
+  *out = &P;
+  return CTXB_OK;
+}
+
+// CTXB_WATCHER: launch the watcher warp of run r's current launch on the
+// library's signal stream and make the victim's stream wait until it runs.
+int launch_watcher(ctxb_run* r) {
+  Probe* P = nullptr;
+  {
+    std::lock_guard<std::mutex> g(probe_mu);
+    if (int rc = probe_module(r->ctx, &P)) return rc;
+  }
+  Driver& d = driver();
+  // the watcher's "started" word: in the drain-notice page (its counter is at
+  // offset 0), away from the gather words that a resume launch resets
+  CUdeviceptr hw = r->hflag_dev + 32, flag = r->flag, started = r->flag + r->rep_off - FLAG_STRIDE + 128,
+              stamp = r->stamps_watch;
+  uint32_t seq = r->gate_seq, sig = r->sig;
+  unsigned long long rep = r->rep_off;
+  void* a[] = {&hw, &seq, &flag, &rep, &sig, &started, &stamp};
+  CU(d.cuLaunchKernel(P->watch, 1, 1, 1, 32, 1, 1, 0, r->arm, a, nullptr));
+  CU(d.cuStreamWaitValue32(r->stream, started, seq, CU_STREAM_WAIT_VALUE_GEQ));
+  r->watching = true;
+  return CTXB_OK;
+}
+
+// Restore-floor probe: generated per slot size, like a restore stub --
+// straight-line evict-first v4 loads of every 512 B group (lane l's 16 B at
+// +16 l) and v1 loads of the 1-3 trailing 128 B rows, all issued before any
+// value is used, then an XOR reduction; stamps {entry, all loads back}.
+std::string floor_src(uint32_t slot) {
+  std::ostringstream o;
+  const uint32_t ng = slot / 512, nt = (slot % 512) / 128;
+  o << "typedef unsigned int u32; typedef unsigned long long u64;\n"
+       "static __device__ __forceinline__ u64 gt() { u64 t; asm volatile(\"mov.u64 %0, %%globaltimer;\" : \"=l\"(t)); return t; }\n"
+       "extern \"C\" __global__ void ctxb_probe_read(const unsigned char* ctx, u64* st, u32* out, u32 zero) {\n"
+       "  const u32 lane = threadIdx.x & 31u, gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;\n"
+       "  const u64 t0 = gt();\n"
+       "  const unsigned char* p = ctx + (u64)gw * " << slot << "ull;\n";
+  for (uint32_t g = 0; g < ng; g++)
+    o << "  const uint4 q" << g << " = __ldcs(reinterpret_cast<const uint4*>(p + " << g * 512 << "u) + lane);\n";
+  for (uint32_t t = 0; t < nt; t++)
+    o << "  const u32 r" << t << " = __ldcs(reinterpret_cast<const u32*>(p + " << ng * 512 + t * 128 << "u) + lane);\n";
+  o << "  u32 acc = 0u";
+  for (uint32_t g = 0; g < ng; g++) o << " ^ q" << g << ".x ^ q" << g << ".y ^ q" << g << ".z ^ q" << g << ".w";
+  for (uint32_t t = 0; t < nt; t++) o << " ^ r" << t;
+  o << ";\n  acc = __reduce_xor_sync(0xffffffffu, acc);\n"
+       "  u64 t1 = 0;\n  if ((acc & zero) == 0u) t1 = gt();\n"
+       "  if (lane == 0u) { st[(u64)gw * 2] = t0; st[(u64)gw * 2 + 1] = t1; out[gw] = acc; }\n}\n";
+  return o.str();
+}
+
+int floor_kernel(CUcontext c, uint32_t slot, CUfunction* fn) {
+  static std::map<std::pair<CUcontext, uint32_t>, CUfunction> cache;
+  auto it = cache.find({c, slot});
+  if (it != cache.end()) {
+    *fn = it->second;
+    return CTXB_OK;
+  }
+  Nvrtc& n = nvrtc();
+  if (!n.ok) return fail(CTXB_E_NVRTC, n.err);
+  std::string src = floor_src(slot);
+  void* prog = nullptr;
+  if (n.CreateProgram(&prog, src.c_str(), "floor.cu", 0, nullptr, nullptr)) return fail(CTXB_E_NVRTC, "floor probe");
+  const char* opts[] = {"--gpu-architecture=sm_100a"};
+  if (n.CompileProgram(prog, 1, opts)) {
+    n.DestroyProgram(&prog);
+    return fail(CTXB_E_NVRTC, "floor probe compile");
+  }
+  size_t cs = 0;
+  n.GetCUBINSize(prog, &cs);
+  std::vector<char> cubin(cs);
+  n.GetCUBIN(prog, cubin.data());
+  n.DestroyProgram(&prog);
+  Driver& d = driver();
+  CUmodule mod = nullptr;
+  CU(d.cuModuleLoadData(&mod, cubin.data()));
+  CU(d.cuModuleGetFunction(fn, mod, "ctxb_probe_read"));
+  cache[{c, slot}] = *fn;
+  return CTXB_OK;
+}
+
 int launch(ctxb_run* r, bool resume) {
   r->sig = ++r->sig_seq;
   if (r->sig == 0) r->sig = ++r->sig_seq;   // 0 is the flags' initial value
@@ -416,6 +570,10 @@ int launch(ctxb_run* r, bool resume) {
   pack_params(r, r->prog, blob);
   void* args[] = {blob.data()};
   Driver& d = driver();
+  if (r->prog->opt.flags & CTXB_WATCHER) {
+    r->gate_seq = (r->gate_seq + 1) & 0x7FFFFFFFu;
+    if (int rc = launch_watcher(r)) return rc;
+  }
   CU(d.cuEventRecord(r->ev0, r->stream));
   CU(d.cuLaunchKernel(resume ? r->mod.resume : r->mod.run, r->grid, 1, 1, (unsigned)r->prog->prog.block, 1, 1, 0,
                       r->stream, args, nullptr));
@@ -503,7 +661,9 @@ int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb
   if (!ir_text || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   *out = nullptr;
   ctxb_options o = opts ? *opts : ctxb_options{CTXB_ALL, CTXB_MODE_CTXBACK, CTXB_POLL_EVERY_INSTR, 8, 0, 1, 0, 8, 512, 0, 1};
-  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 32767 || ((o.flags & 2048u) && (o.flags & 4096u)) || o.flag_depth > 8 || o.load_every > 1024 || o.min_blocks_per_sm > 32)
+  if (o.mode > 3 || o.poll_policy > 2 || o.flags > 65535 || ((o.flags & 2048u) && (o.flags & 4096u)) ||
+      ((o.flags & CTXB_ARMED_SIGNAL) && (o.flags & CTXB_WATCHER)) || o.flag_depth > 8 || o.load_every > 1024 ||
+      o.min_blocks_per_sm > 32)
     return fail(CTXB_E_INVALID_ARG, "bad options");
   std::unique_ptr<ctxb_program> p(new ctxb_program);
   p->opt = Options{o.flags, o.mode, o.poll_policy, o.poll_every ? o.poll_every : 8, o.debug,
@@ -661,6 +821,43 @@ int ctxb_occupancy(ctxb_program* p, uint32_t* bps, uint32_t* nsm) {
   return CTXB_OK;
 }
 
+int ctxb_persistent_grid(ctxb_program* p, uint32_t* grid) {
+  if (!p || !grid) return fail(CTXB_E_INVALID_ARG, "NULL argument");
+  uint32_t bps = 0, nsm = 0;
+  if (int rc = ctxb_occupancy(p, &bps, &nsm)) return rc;
+  *grid = bps * nsm;
+  if (!(p->opt.flags & CTXB_WATCHER) || bps == 0) return CTXB_OK;
+  // the watcher warp (32 threads, its registers, no shared memory) must fit
+  // on one SM next to bps blocks, else that SM hosts one block fewer
+  CUcontext c;
+  if (int rc = ensure_ctx(&c)) return rc;
+  Probe* P = nullptr;
+  {
+    std::lock_guard<std::mutex> g(probe_mu);
+    if (int rc = probe_module(c, &P)) return rc;
+  }
+  Mod m;
+  if (int rc = ensure_module(p, c, &m)) return rc;
+  Driver& d = driver();
+  int rw = 0, rv = 0, rr = 0, sv = 0, sr = 0, smem_sm = 0, maxw = 0;
+  CUdevice dev;
+  CU(d.cuCtxGetDevice(&dev));
+  CU(d.cuFuncGetAttribute(&rw, CU_FUNC_ATTRIBUTE_NUM_REGS, P->watch));
+  CU(d.cuFuncGetAttribute(&rv, CU_FUNC_ATTRIBUTE_NUM_REGS, m.run));
+  CU(d.cuFuncGetAttribute(&rr, CU_FUNC_ATTRIBUTE_NUM_REGS, m.resume));
+  CU(d.cuFuncGetAttribute(&sv, CU_FUNC_ATTRIBUTE_SHARED_SIZE_BYTES, m.run));
+  CU(d.cuFuncGetAttribute(&sr, CU_FUNC_ATTRIBUTE_SHARED_SIZE_BYTES, m.resume));
+  CU(d.cuDeviceGetAttribute(&smem_sm, CU_DEVICE_ATTRIBUTE_MAX_SHARED_MEMORY_PER_MULTIPROCESSOR, dev));
+  CU(d.cuDeviceGetAttribute(&maxw, CU_DEVICE_ATTRIBUTE_MAX_THREADS_PER_MULTIPROCESSOR, dev));
+  auto warp_regs = [](int r) { return ((r * 32 + 255) / 256) * 256; };
+  const uint32_t wpb = p->prog.block / 32;
+  const uint64_t regs = (uint64_t)bps * wpb * (uint64_t)warp_regs(std::max(rv, rr)) + warp_regs(rw);
+  const uint64_t warps = (uint64_t)bps * wpb + 1;
+  const uint64_t smem = (uint64_t)bps * (uint64_t)(std::max(sv, sr) + 1024);
+  if (regs > 65536 || warps > (uint64_t)maxw / 32 || bps + 1 > 32 || smem > (uint64_t)smem_sm) *grid -= 1;
+  return CTXB_OK;
+}
+
 int ctxb_context_capacity(const ctxb_program* p, uint32_t grid, uint64_t* bytes) {
   if (!p || !bytes || grid == 0) return fail(CTXB_E_INVALID_ARG, "bad argument");
   if (p->opt.mode == CTXB_MODE_FULL_HW && p->num_regs == 0)
@@ -735,7 +932,7 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
     // (+ one page for the drain-notice exit counter, just below the replicas)
     r->rep_off = ((256 + (uint64_t)grid * 4 + FLAG_STRIDE - 1) / FLAG_STRIDE) * FLAG_STRIDE + FLAG_STRIDE;
     CU(d.cuMemAlloc(&f, r->rep_off + (size_t)FLAG_REPLICAS * FLAG_STRIDE));
-    CU(d.cuMemAlloc(&s, (size_t)r->n_warps * 32));
+    CU(d.cuMemAlloc(&s, (size_t)r->n_warps * 32 + 64));   // + the watcher's stamp
     CU(d.cuMemAlloc(&t, (size_t)r->n_warps * 4));
     r->flag = f;
     r->stamps = s;
@@ -754,7 +951,8 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
     r->hflag = h;
     CU(d.cuMemHostGetDevicePointer(&r->hflag_dev, h, 0));
   }
-  if ((p->opt.flags & CTXB_ARMED_SIGNAL) && !r->arm) {
+  r->stamps_watch = r->stamps + (CUdeviceptr)r->n_warps * 32;
+  if ((p->opt.flags & (CTXB_ARMED_SIGNAL | CTXB_WATCHER)) && !r->arm) {
     int lo = 0, hi = 0;
     CU(d.cuCtxGetStreamPriorityRange(&lo, &hi));
     CU(d.cuStreamCreateWithPriority(&r->arm, CU_STREAM_NON_BLOCKING, hi));
@@ -809,8 +1007,17 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     *hf = 1u;
     std::atomic_thread_fence(std::memory_order_seq_cst);
   }
-  // test knob: CTXB_HOST_SIGNAL_ONLY=1 drops the fallback, so the relay is the only path
-  const char* ho = hf ? getenv("CTXB_HOST_SIGNAL_ONLY") : nullptr;
+  // CTXB_WATCHER: the co-resident watcher warp sees this store over PCIe and
+  // raises the device flags; the stream memory op stays as the fallback
+  const bool watch = r->watching;
+  if (watch) {
+    *(static_cast<volatile uint32_t*>(r->hflag) + 8) = r->gate_seq;
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    r->watching = false;
+  }
+  // test knob: CTXB_HOST_SIGNAL_ONLY=1 drops the fallback, so the relay (or
+  // the watcher) is the only path
+  const char* ho = (hf || watch) ? getenv("CTXB_HOST_SIGNAL_ONLY") : nullptr;
   const bool host_only = ho && atoi(ho) != 0;
   CUstream cs = (CUstream)ctrl;
   if (r->armed) {
@@ -821,7 +1028,7 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     cs = r->arm;
   } else {
     CU(d.cuEventRecord(r->evf, cs));
-    if (!(hf && host_only))
+    if (!((hf || watch) && host_only))
       if (int rc = write_signal(r, cs)) return rc;
   }
   // env CTXB_PREEMPT_TIMEOUT_US > 0: give up waiting for the drain after that
@@ -880,8 +1087,8 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     st->latency_us = st->warps_preempted ? (double)(tmax - tmin) * 1e-3 : 0.0;
     float ms = 0;
     CU(d.cuEventElapsedTime(&ms, r->evf, r->ev1));
-    // with CTXB_HOST_SIGNAL the signal is the host store, which the event does not bound
-    st->signal_to_drained_us = hf ? 0.0 : (double)ms * 1e3;
+    // with CTXB_HOST_SIGNAL / CTXB_WATCHER the signal is the host store, which the event does not bound
+    st->signal_to_drained_us = (hf || watch) ? 0.0 : (double)ms * 1e3;
   }
   return CTXB_OK;
 }
@@ -894,6 +1101,11 @@ int ctxb_preempt_async(ctxb_run* r, void* ctrl) {
   if (r->prog->opt.flags & CTXB_HOST_SIGNAL) {   // lowered when the launch is collected
     *static_cast<volatile uint32_t*>(r->hflag) = 1u;
     std::atomic_thread_fence(std::memory_order_seq_cst);
+  }
+  if (r->watching) {   // CTXB_WATCHER: the watcher relays the host store (the memop stays as the fallback)
+    *(static_cast<volatile uint32_t*>(r->hflag) + 8) = r->gate_seq;
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    r->watching = false;
   }
   if (r->armed) {
     *(static_cast<volatile uint32_t*>(r->hflag) + 16) = r->gate_seq;
@@ -972,110 +1184,7 @@ int ctxb_query(ctxb_run* r, int* running) {
 }
 
 // ---- flag propagation probe (measured separately) -------------
-namespace {
-const char* kProbeSrc = R"CUDA(
-typedef unsigned int u32; typedef unsigned long long u64;
-static __device__ __forceinline__ u64 gt() { u64 t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); return t; }
-static __device__ __forceinline__ u32 ldcv(const u32* p) { u32 v; asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p)); return v; }
-extern "C" __global__ void ctxb_probe_spin(const u32* flag, u64* out) {
-  u64 t0 = gt();
-  while (ldcv(flag) == 0u) { if (gt() - t0 > 20000000ull) break; }   // 20 ms timeout
-  if (threadIdx.x == 0) out[1] = gt();
-}
-extern "C" __global__ void ctxb_probe_stamp(u64* out) { if (threadIdx.x == 0) out[0] = gt(); }
-)CUDA";
 
-struct Probe {
-  CUmodule mod = nullptr;
-  CUfunction spin = nullptr, stamp = nullptr;
-};
-
-std::mutex probe_mu;
-
-// The probe module of context c (compiled once with NVRTC); caller holds probe_mu.
-int probe_module(CUcontext c, Probe** out) {
-  static std::map<CUcontext, Probe> probes;
-  Probe& P = probes[c];
-  Driver& d = driver();
-  if (!P.mod) {
-    Nvrtc& n = nvrtc();
-    if (!n.ok) return fail(CTXB_E_NVRTC, n.err);
-    void* prog = nullptr;
-    if (n.CreateProgram(&prog, kProbeSrc, "probe.cu", 0, nullptr, nullptr)) return fail(CTXB_E_NVRTC, "probe");
-    const char* opts[] = {"--gpu-architecture=sm_100a"};
-    if (n.CompileProgram(prog, 1, opts)) {
-      n.DestroyProgram(&prog);
-      return fail(CTXB_E_NVRTC, "probe compile");
-    }
-    size_t cs = 0;
-    n.GetCUBINSize(prog, &cs);
-    std::vector<char> cubin(cs);
-    n.GetCUBIN(prog, cubin.data());
-    n.DestroyProgram(&prog);
-    CU(d.cuModuleLoadData(&P.mod, cubin.data()));
-    CU(d.cuModuleGetFunction(&P.spin, P.mod, "ctxb_probe_spin"));
-    CU(d.cuModuleGetFunction(&P.stamp, P.mod, "ctxb_probe_stamp"));
-  }
-  *out = &P;
-  return CTXB_OK;
-}
-
-// Restore-floor probe: generated per slot size, like a restore stub --
-// straight-line evict-first v4 loads of every 512 B group (lane l's 16 B at
-// +16 l) and v1 loads of the 1-3 trailing 128 B rows, all issued before any
-// value is used, then an XOR reduction; stamps {entry, all loads back}.
-std::string floor_src(uint32_t slot) {
-  std::ostringstream o;
-  const uint32_t ng = slot / 512, nt = (slot % 512) / 128;
-  o << "typedef unsigned int u32; typedef unsigned long long u64;\n"
-       "static __device__ __forceinline__ u64 gt() { u64 t; asm volatile(\"mov.u64 %0, %%globaltimer;\" : \"=l\"(t)); return t; }\n"
-       "extern \"C\" __global__ void ctxb_probe_read(const unsigned char* ctx, u64* st, u32* out, u32 zero) {\n"
-       "  const u32 lane = threadIdx.x & 31u, gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;\n"
-       "  const u64 t0 = gt();\n"
-       "  const unsigned char* p = ctx + (u64)gw * " << slot << "ull;\n";
-  for (uint32_t g = 0; g < ng; g++)
-    o << "  const uint4 q" << g << " = __ldcs(reinterpret_cast<const uint4*>(p + " << g * 512 << "u) + lane);\n";
-  for (uint32_t t = 0; t < nt; t++)
-    o << "  const u32 r" << t << " = __ldcs(reinterpret_cast<const u32*>(p + " << ng * 512 + t * 128 << "u) + lane);\n";
-  o << "  u32 acc = 0u";
-  for (uint32_t g = 0; g < ng; g++) o << " ^ q" << g << ".x ^ q" << g << ".y ^ q" << g << ".z ^ q" << g << ".w";
-  for (uint32_t t = 0; t < nt; t++) o << " ^ r" << t;
-  o << ";\n  acc = __reduce_xor_sync(0xffffffffu, acc);\n"
-       "  u64 t1 = 0;\n  if ((acc & zero) == 0u) t1 = gt();\n"
-       "  if (lane == 0u) { st[(u64)gw * 2] = t0; st[(u64)gw * 2 + 1] = t1; out[gw] = acc; }\n}\n";
-  return o.str();
-}
-
-int floor_kernel(CUcontext c, uint32_t slot, CUfunction* fn) {
-  static std::map<std::pair<CUcontext, uint32_t>, CUfunction> cache;
-  auto it = cache.find({c, slot});
-  if (it != cache.end()) {
-    *fn = it->second;
-    return CTXB_OK;
-  }
-  Nvrtc& n = nvrtc();
-  if (!n.ok) return fail(CTXB_E_NVRTC, n.err);
-  std::string src = floor_src(slot);
-  void* prog = nullptr;
-  if (n.CreateProgram(&prog, src.c_str(), "floor.cu", 0, nullptr, nullptr)) return fail(CTXB_E_NVRTC, "floor probe");
-  const char* opts[] = {"--gpu-architecture=sm_100a"};
-  if (n.CompileProgram(prog, 1, opts)) {
-    n.DestroyProgram(&prog);
-    return fail(CTXB_E_NVRTC, "floor probe compile");
-  }
-  size_t cs = 0;
-  n.GetCUBINSize(prog, &cs);
-  std::vector<char> cubin(cs);
-  n.GetCUBIN(prog, cubin.data());
-  n.DestroyProgram(&prog);
-  Driver& d = driver();
-  CUmodule mod = nullptr;
-  CU(d.cuModuleLoadData(&mod, cubin.data()));
-  CU(d.cuModuleGetFunction(fn, mod, "ctxb_probe_read"));
-  cache[{c, slot}] = *fn;
-  return CTXB_OK;
-}
-}  // namespace
 
 int ctxb_restore_floor(void* stream, uint32_t bytes_per_warp, uint32_t grid_blocks, uint32_t block,
                        uint32_t trials, double* median_us) {

@@ -14,7 +14,7 @@ import numpy as np
 
 __all__ = [
     "LIB_PATH", "CtxbError", "lib",
-    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "GATHER_RESUME", "SYNC_POLL", "HOST_SIGNAL", "ARMED_SIGNAL", "OSRB_SMEM", "OSRB_LANES", "FLAG_REPLICAS", "DRAIN_NOTICE", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
+    "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "GATHER_RESUME", "SYNC_POLL", "HOST_SIGNAL", "ARMED_SIGNAL", "OSRB_SMEM", "OSRB_LANES", "FLAG_REPLICAS", "DRAIN_NOTICE", "WATCHER", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
     "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS", "DEBUG_NO_AUTO_GATHER", "DEBUG_NO_FP_SHARE",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "E_TIMEOUT", "EXPORTED_SYMBOLS",
@@ -28,6 +28,7 @@ LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libctxb.so"
 RELAXED, REVERT, OSRB, ALL, DEFER, PRUNE, RANK_RESUME, EXACT, GATHER_RESUME, SYNC_POLL, HOST_SIGNAL = \
     1, 2, 4, 7, 8, 16, 32, 64, 128, 256, 512
 ARMED_SIGNAL, OSRB_SMEM, OSRB_LANES, FLAG_REPLICAS, DRAIN_NOTICE = 1024, 2048, 4096, 8192, 16384
+WATCHER = 32768
 MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
 DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1, 2, 4, 8, 16
@@ -42,6 +43,7 @@ EXPORTED_SYMBOLS = [
     "ctxb_occupancy", "ctxb_context_capacity", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait",
     "ctxb_query", "ctxb_flag_propagation", "ctxb_launch_ms", "ctxb_resume_stats_get", "ctxb_context_bytes", "ctxb_read_headers", "ctxb_read_stamps",
     "ctxb_run_destroy", "ctxb_preempt_async", "ctxb_program_cubin", "ctxb_restore_floor",
+    "ctxb_persistent_grid",
 ]
 
 
@@ -120,6 +122,7 @@ def _load():
         "ctxb_preempt_async": (I, [P, P]),
         "ctxb_program_cubin": (I, [P, P, SZ, C.POINTER(SZ)]),
         "ctxb_restore_floor": (I, [P, U32, U32, U32, U32, C.POINTER(C.c_double)]),
+        "ctxb_persistent_grid": (I, [P, C.POINTER(U32)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -282,6 +285,13 @@ class Program:
         a, n = C.c_uint32(), C.c_uint32()
         _chk(lib.ctxb_occupancy(self._h, C.byref(a), C.byref(n)))
         return a.value, n.value
+
+    def persistent_grid(self):
+        """Blocks of a persistent grid (ctxb_persistent_grid): every block
+        resident at once, room left for the CTXB_WATCHER warp."""
+        g = C.c_uint32()
+        _chk(lib.ctxb_persistent_grid(self._h, C.byref(g)))
+        return g.value
 
     def context_capacity(self, grid):
         b = C.c_uint64()

@@ -255,3 +255,17 @@ def test_gather_resume_default_for_atomics():
                           ).info["gather_resume"] == 0
         assert cb.Program(txt, poll_policy=pol, flags=cb.ALL | cb.GATHER_RESUME,
                           debug=cb.DEBUG_NO_COMPILE).info["gather_resume"] == 1
+
+
+def test_watcher_option_validation():
+    """CTXB_WATCHER and CTXB_ARMED_SIGNAL both use the library's signal stream:
+    exclusive.  The watcher changes no plan and no generated kernel."""
+    from workloads import configs
+    txt = configs.c2(128, 128, 64)["ir"]
+    with pytest.raises(cb.CtxbError) as e:
+        cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | cb.WATCHER | cb.ARMED_SIGNAL,
+                   debug=cb.DEBUG_NO_COMPILE)
+    assert e.value.code == -1
+    a = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | cb.WATCHER, debug=cb.DEBUG_NO_COMPILE)
+    b = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
+    assert a.source == b.source

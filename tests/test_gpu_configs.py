@@ -218,7 +218,10 @@ def test_c2s_full_flag_equals_c2():
                                         ("c3", "replicas"), ("c2", "replicas"), ("c3", "load4"),
                                         ("c3", "replicas+load4"), ("c3r2", "load4"),
                                         ("c3r2", "combo"), ("c2", "combo"), ("c4a", "combo"), ("c4a", False),
-                                        ("c2", "notice"), ("c3r2", "notice"), ("c2s", "notice")])
+                                        ("c2", "notice"), ("c3r2", "notice"), ("c2s", "notice"),
+                                        ("c2", "watcher"), ("c3b", "watcher"), ("c4a", "watcher"), ("c2s", "watcher"),
+                                        ("c2", "watcher_only"), ("c3b", "watcher_only"), ("c2", "watcher_gather"),
+                                        ("c3b", "watcher_gather")])
 def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     """random flag times, repeated and nested
     preempt -> resume -> preempt ... cycles (each resume can be preempted
@@ -230,7 +233,10 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     CTXB_ARMED_SIGNAL, every launch and resume pre-enqueues its signal behind
     a host gate; runs that end unpreempted are disarmed.
     "replicas" / "load4": CTXB_FLAG_REPLICAS (master pollers forward the
-    signal to 64 replicas) and loads at every 4th poll visit."""
+    signal to 64 replicas) and loads at every 4th poll visit.
+    "watcher": CTXB_WATCHER (+ drain notice) -- a co-resident warp relays the
+    host store; "watcher_only": without the memop fallback, so
+    every preemption arrives through the watcher."""
     import time
     import torch
     cb = _cb()
@@ -238,8 +244,8 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
         cfg = configs.c4a(1 << 28, grid=1)
         bufs = [to_dev(cfg["buffers"]["keys"]), to_dev(cfg["buffers"]["starts"]), None]
         out_i, mb = 2, 0
-    elif which in ("c3", "c3r2"):
-        cfg = configs.c3(rows_per_iter=2 if which == "c3r2" else 1)
+    elif which in ("c3", "c3r2", "c3b"):
+        cfg = configs.c3(**configs.BENCH_C3) if which == "c3b" else configs.c3(rows_per_iter=2 if which == "c3r2" else 1)
         bufs = [to_dev(cfg["buffers"]["X"]), torch.zeros(cfg["W"] * cfg["H"], dtype=torch.int32, device="cuda")]
         out_i, mb = 1, 0
     else:
@@ -247,7 +253,7 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
         bufs = [to_dev(cfg["buffers"]["A"]), to_dev(cfg["buffers"]["B"]),
                 torch.zeros(4096 * 4096, dtype=torch.int32, device="cuda")]
         out_i, mb = 2, 2
-    if host is True:
+    if host is True or host == "watcher_only":
         monkeypatch.setenv("CTXB_HOST_SIGNAL_ONLY", "1")
     # "combo": the runtime options together (armed signal, gathered resume, flag
     # replicas, sparse flag loads; C4a also the synchronous test and shared-memory OSRB slots)
@@ -256,11 +262,15 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
         combo |= cb.SYNC_POLL | cb.OSRB_SMEM
     extra = {"armed": cb.ARMED_SIGNAL, "replicas": cb.FLAG_REPLICAS, "load4": 0, "combo": combo,
              "notice": cb.DRAIN_NOTICE | cb.ARMED_SIGNAL,
+             "watcher": cb.WATCHER | cb.DRAIN_NOTICE, "watcher_only": cb.WATCHER,
+             "watcher_gather": cb.WATCHER | cb.DRAIN_NOTICE | cb.GATHER_RESUME,
              "replicas+load4": cb.FLAG_REPLICAS, True: cb.HOST_SIGNAL, False: 0}[host]
     prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=mb, flags=cb.ALL | extra,
                       load_every=4 if host in ("load4", "replicas+load4", "combo") else 1)
-    bps, nsm = prog.occupancy()
-    grid = bps * nsm
+    grid = prog.persistent_grid()
+    if host in ("watcher", "watcher_only", "watcher_gather") and which in ("c2", "c2s"):
+        bps, nsm = prog.occupancy()
+        assert grid == bps * nsm - 1      # the full register file leaves no room for the watcher warp
     if bufs[out_i] is None:
         bufs[out_i] = torch.zeros(256 * grid, dtype=torch.int32, device="cuda")
     ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")

@@ -116,10 +116,14 @@ def c4b(trials):
     ctx = torch.empty(base.context_capacity(grid), dtype=torch.uint8, device="cuda")
     bfs(base, grid, ctx)
     t0 = float(np.median([bfs(base, grid, ctx)[0] for _ in range(5)]))
-    for polls in ("both", "vertex", "edge"):
+    variants = [(p, f, le) for p in ("both", "vertex", "edge") for f in ("word", "replicas") for le in (1, 4)]
+    if os.environ.get("C4B_VARIANTS"):      # e.g. "edge:replicas:1,edge:replicas:2"
+        variants = [(a, b, int(c)) for a, b, c in (v.split(":") for v in os.environ["C4B_VARIANTS"].split(","))]
+    for polls, fname, le in variants:
         txt = configs.c4b_ir(polls)
-        for fname, fl in (("word", 0), ("replicas", cb.FLAG_REPLICAS)):
-            for le in (1, 4):
+        fl = {"word": 0, "replicas": cb.FLAG_REPLICAS}[fname]
+        if True:
+            if True:
                 prog = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | fl, load_every=le)
                 ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
                 _, _, sizes = bfs(prog, grid, ctx)
