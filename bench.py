@@ -1419,7 +1419,7 @@ def compact_line(d, detail_path):
     cpu = d.get("cpu_baseline")
     if cpu:
         cpu = {"value": _r(cpu["value"], 1), "unit": cpu["unit"], "cores": cpu["cores"], "kind": "oracle",
-               "sample": "C2 IR 256^3, TB0, 8 warps, 1 poll visit"}
+               "sample": "C2 256^3, TB0 (8 warps), 1 poll"}
     e = d["e2e"]
     cfgs = {}
     for k, c in d.get("configs", {}).items():
@@ -1439,9 +1439,9 @@ def compact_line(d, detail_path):
         "metric": d["metric"], "value": d["value"], "unit": d["unit"], "n_gpus": d["n_gpus"], "steps": d["steps"],
         "warmup": d["warmup"], "ms_per_step": d["ms_per_step"], "higher_is_better": False, "scaling": "weak",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": f"C2 SGEMM IR {d['config']['size']}^3 (configs[1]), {d['config']['grid']}x256 "
-                               "persistent, flag U[.05,.95]T",
-                   "l2": "inputs > L2; resume L2-cold" if "cold" in d["config"]["resume_l2"] else "inputs > L2; resume warm"},
+        "config": {"workload": f"C2 SGEMM IR {d['config']['size']}^3 (configs[1]), {d['config']['grid']}x256, "
+                               "flag U[.05,.95]T",
+                   "l2": "inputs>L2, cold resume" if "cold" in d["config"]["resume_l2"] else "inputs>L2, warm resume"},
         "routines_us": _r(m["latency_us_median"], 3), "resume_us": _r(m["resume_us_median"], 3),
         "context_bytes_per_tb": m.get("context_bytes_per_tb"),
         "signal": d["signal"],
