@@ -338,21 +338,11 @@ def bulk_bandwidth(cb, mib, reps=5):
 
 
 def poll_overhead(cb, size, grid, bufs, reps=20):
-    import torch
-    out = {}
-    for name, dbg in (("polls", 0), ("no_polls", cb.DEBUG_NO_POLLS)):
-        prog = make_c2(cb, size, cb.MODE_CTXBACK, dbg)
-        ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
-        ts = []
-        for i in range(reps + 1):
-            run = prog.launch(grid, list(bufs), [], ctx)
-            run.wait()
-            if i:
-                ts.append(run.launch_ms())
-            del run
-        out[name] = float(np.median(ts))
-    out["overhead_pct"] = 100.0 * (out["polls"] / out["no_polls"] - 1.0)
-    return out
+    """C2's poll-site overhead: interleaved launches of the polled kernel and
+    the same kernel without polls, on the polled kernel's own persistent grid."""
+    from workloads import configs
+    return _poll_overhead(cb, configs.c2_ir(size, size, size, polls="iter"), None, lambda: list(bufs),
+                          min_blocks=2, reps=reps)
 
 
 def one_direction_peaks(gib=2, reps=5):
@@ -482,9 +472,10 @@ def poll_tuning(cb, config):
 
 
 def _progs(cb, ir_text, debug=0, min_blocks=0, extra_flags=0, load_every=1):
+    """Every mode of a config, on the headline's signal path (--signal)."""
     return {name: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT if "poll" in ir_text else cb.POLL_EVERY_INSTR,
-                             mode=mode, flags=flags | extra_flags, debug=debug | dbg, min_blocks_per_sm=min_blocks,
-                             load_every=load_every)
+                             mode=mode, flags=flags | extra_flags | SIGNAL_FLAGS, debug=debug | dbg,
+                             min_blocks_per_sm=min_blocks, load_every=load_every)
             for name, mode, flags, dbg in _modes(ir_text)}
 
 
@@ -550,6 +541,9 @@ def _poll_overhead(cb, ir_text, grid, make_bufs, uniforms=(), extra_flags=0, min
     for name, dbg in (("polls_ms", 0), ("no_polls_ms", cb.DEBUG_NO_POLLS)):
         progs[name] = cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | extra_flags, debug=dbg,
                                  min_blocks_per_sm=min_blocks, load_every=load_every)
+    if grid is None:   # the polled kernel's own persistent grid (no watcher: the signal path is not the poll's cost)
+        grid = progs["polls_ms"].persistent_grid()
+    for name in progs:
         ctxs[name] = torch.empty(progs[name].context_capacity(grid), dtype=torch.uint8, device="cuda")
         ts[name] = []
     for i in range(reps + 1):
@@ -561,6 +555,7 @@ def _poll_overhead(cb, ir_text, grid, make_bufs, uniforms=(), extra_flags=0, min
             del run
     out = {name: float(np.median(v)) for name, v in ts.items()}
     out["overhead_pct"] = 100.0 * (out["polls_ms"] / out["no_polls_ms"] - 1.0)
+    out["grid"] = grid
     return out
 
 
@@ -649,7 +644,7 @@ def bench_c2s(cb, trials, seed):
     res = _flag_trials(progs, grid, make, [], lambda b_: bool(torch.equal(b_[2], ref)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
     res["static"]["smem_bytes_per_tb"] = 4 * 2048
-    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], progs["ctxback"].persistent_grid(), make, min_blocks=2)
+    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], None, make, min_blocks=2)
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
@@ -683,8 +678,7 @@ def bench_c3(cb, trials, seed):
     fr = np.random.default_rng(seed + 2).uniform(0.05, 0.95, trials)
     res = _flag_trials(progs, grid, make, [], lambda b: bool(torch.equal(b[1], ref)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
-    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], progs["ctxback"].persistent_grid(), make,
-                                          **poll_tuning(cb, "c3"))
+    res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], None, make, **poll_tuning(cb, "c3"))
     res["reduction_vs_full_hw"] = _reduction(res)
     res["rank_resume_reduction_vs_full_hw"] = _reduction(res, "ctxback_rank_resume")
     res["gather_reduction_vs_full_hw_gather"] = _reduction(res, "ctxback_gather", "full_hw_gather")
@@ -724,7 +718,8 @@ def bench_c4a(cb, trials, seed):
     fr = np.random.default_rng(seed + 3).uniform(0.05, 0.95, trials)
     res = _flag_trials(progs, grid, make, [], lambda b: bool(torch.equal(hsum(b[2]), want)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
-    g_own = progs["ctxback"].persistent_grid()   # the CTXBack kernel's own persistent grid
+    g_own = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | poll_tuning(cb, "c4a")["extra_flags"],
+                       ).persistent_grid()   # the polled kernel's own persistent grid
     if g_own > grid:
         dH = torch.zeros(256 * g_own, dtype=torch.int32, device="cuda")
     res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], g_own, make, **poll_tuning(cb, "c4a"))   # incl. the OSRB copy
@@ -824,7 +819,7 @@ def bench_c4b(cb, trials, seed):
                            flags=cb.ALL | poll_tuning(cb, "c4b").get("extra_flags", 0))
            for key, dbg in (("polls_ms", 0), ("no_polls_ms", cb.DEBUG_NO_POLLS))}
     tv = {key: [] for key in prs}
-    g_own = prs["polls_ms"].persistent_grid()   # the CTXBack kernel's own persistent grid
+    g_own = prs["polls_ms"].persistent_grid()   # the polled kernel's own persistent grid (no watcher)
     for i in range(10):                       # interleaved: drift hits both alike
         for key, pr in prs.items():
             t_ = bfs_ms(pr, g_own)
