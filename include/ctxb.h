@@ -438,7 +438,9 @@ int ctxb_context_bytes(const ctxb_run* run, uint64_t* payload, uint64_t* header,
  * (4 u32 per warp) of the last completed launch into host memory. */
 int ctxb_read_headers(const ctxb_run* run, uint32_t* host_out, uint64_t n_words);
 /* Copy the per-warp %globaltimer stamps {t_flag_seen, t_saved, t_resume_entry,
- * t_site_reached} (4 u64 per warp). */
+ * t_site_reached} (4 u64 per warp).  With n_words > 4 x warps one more word
+ * follows: the %globaltimer at which the run's CTXB_WATCHER warp last raised
+ * the flag (0 if it never did). */
 int ctxb_read_stamps(const ctxb_run* run, uint64_t* host_out, uint64_t n_words);
 
 /* Release the run handle; its device resources return to the program's pool.

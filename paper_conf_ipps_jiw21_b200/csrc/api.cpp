@@ -933,6 +933,7 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
     r->rep_off = ((256 + (uint64_t)grid * 4 + FLAG_STRIDE - 1) / FLAG_STRIDE) * FLAG_STRIDE + FLAG_STRIDE;
     CU(d.cuMemAlloc(&f, r->rep_off + (size_t)FLAG_REPLICAS * FLAG_STRIDE));
     CU(d.cuMemAlloc(&s, (size_t)r->n_warps * 32 + 64));   // + the watcher's stamp
+    CU(d.cuMemsetD8Async(s + (CUdeviceptr)r->n_warps * 32, 0, 64, nullptr));
     CU(d.cuMemAlloc(&t, (size_t)r->n_warps * 4));
     r->flag = f;
     r->stamps = s;
@@ -1365,7 +1366,9 @@ int ctxb_read_stamps(const ctxb_run* r, uint64_t* out, uint64_t n) {
   if (!r || !out) return fail(CTXB_E_INVALID_ARG, "NULL argument");
   if (int rc = settle(r)) return rc;
   if (n < (uint64_t)r->n_warps * 4) return fail(CTXB_E_BUFFER_TOO_SMALL, "need 4 words per warp");
-  CU(driver().cuMemcpyDtoH(out, r->stamps, (size_t)r->n_warps * 32));
+  // one more word: the CTXB_WATCHER stamp (when the last watcher raised the flag)
+  const size_t words = (size_t)r->n_warps * 4 + (n > (uint64_t)r->n_warps * 4 ? 1 : 0);
+  CU(driver().cuMemcpyDtoH(out, r->stamps, words * 8));
   return CTXB_OK;
 }
 

@@ -406,3 +406,9 @@ class Run:
         a = np.zeros(self.n_warps * 4, dtype=np.uint64)
         _chk(lib.ctxb_read_stamps(self._h, a.ctypes.data_as(C.POINTER(C.c_uint64)), a.size))
         return a.reshape(-1, 4)
+
+    def watcher_stamp(self):
+        """%globaltimer at which the CTXB_WATCHER warp last raised the flag (0: never)."""
+        a = np.zeros(self.n_warps * 4 + 1, dtype=np.uint64)
+        _chk(lib.ctxb_read_stamps(self._h, a.ctypes.data_as(C.POINTER(C.c_uint64)), a.size))
+        return int(a[-1])

@@ -1,7 +1,8 @@
 """End-to-end preemption timeline on one clock: the host-clock <->
 %globaltimer offset is measured NTP-style by tools/clock_sync_probe (before
-and after, to bound drift), then C2 flag preemptions (armed and memop signal)
-are timed from the host call (CLOCK_REALTIME) through the first warp seeing
+and after, to bound drift), then C2 flag preemptions (armed and memop signal,
+the watcher with and without the drain notice) are timed from the host call
+(CLOCK_REALTIME) through the watcher raising the flag, the first warp seeing
 the signal and the last warp's saved context (device stamps, shifted onto the
 host clock) to ctxb_preempt returning.  GPU; prints a markdown table."""
 import json
@@ -36,12 +37,14 @@ def main():
     c = torch.zeros(4096 * 4096, dtype=torch.int32, device="cuda")
     s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
     res = {}
-    for name, fl in (("armed", cb.ARMED_SIGNAL), ("memop", 0)):
+    for name, fl in (("armed", cb.ARMED_SIGNAL), ("memop", 0), ("watcher", cb.WATCHER),
+                     ("watcher + notice", cb.WATCHER | cb.DRAIN_NOTICE)):
         prog = cb.Program(configs.c2_ir(), poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=2, flags=cb.ALL | fl)
-        ctx = torch.empty(prog.context_capacity(296), dtype=torch.uint8, device="cuda")
+        grid = prog.persistent_grid()
+        ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
         rows = []
         for fr in np.random.default_rng(3).uniform(0.1, 0.9, 16):
-            run = prog.launch(296, [a, b, c], [], ctx, s)
+            run = prog.launch(grid, [a, b, c], [], ctx, s)
             t0 = time.perf_counter()
             while time.perf_counter() < t0 + fr * 5.3e-3:
                 pass
@@ -52,7 +55,9 @@ def main():
             pre = hd[:, 2] == 1
             if pre.any():
                 stp = run.stamps()[pre].astype(np.int64)
-                rows.append((h0, int(stp[:, 0].min()), int(stp[:, 1].max()), h1))
+                w = run.watcher_stamp() if fl & cb.WATCHER else 0
+                rows.append((h0, int(stp[:, 0].min()), int(stp[:, 1].max()), h1, w or int(stp[:, 0].min()),
+                             int(stp[:, 0].max())))
                 run.resume(s)
             run.wait()
             del run
@@ -63,17 +68,21 @@ def main():
         f = (h - o1["host_ns"]) / max(1, o2["host_ns"] - o1["host_ns"])
         return o1["offset_ns"] + f * (o2["offset_ns"] - o1["offset_ns"])
     print(f"offset before / after: {o1} / {o2}")
-    lines = ["| signal | host call -> first warp sees the signal | first seen -> last context saved | "
-             "last saved -> ctxb_preempt returns | host call -> return |", "|---|---|---|---|---|"]
+    lines = ["| signal | host call -> flag raised (watcher) | -> first warp sees the signal | first seen -> last seen | "
+             "first seen -> last context saved | last saved -> ctxb_preempt returns | host call -> return |",
+             "|---|---|---|---|---|---|---|"]
     for name, rows in res.items():
         r = np.array(rows, dtype=np.float64)
         off = np.array([off_at(x) for x in r[:, 0]])
-        a_ = (r[:, 1] - off - r[:, 0]) / 1e3
+        w_ = (r[:, 4] - off - r[:, 0]) / 1e3
+        a_ = (r[:, 1] - r[:, 4]) / 1e3
+        s_ = (r[:, 5] - r[:, 1]) / 1e3
         b_ = (r[:, 2] - r[:, 1]) / 1e3
         c_ = (r[:, 3] - (r[:, 2] - off)) / 1e3
         d_ = (r[:, 3] - r[:, 0]) / 1e3
-        lines.append(f"| {name} | {np.median(a_):.1f} µs | {np.median(b_):.1f} µs | {np.median(c_):.1f} µs | "
-                     f"{np.median(d_):.1f} µs |")
+        wt = f"{np.median(w_):.1f} µs" if "watcher" in name else "—"
+        lines.append(f"| {name} | {wt} | {np.median(a_ if 'watcher' in name else w_ + a_):.1f} µs | "
+                     f"{np.median(s_):.1f} µs | {np.median(b_):.1f} µs | {np.median(c_):.1f} µs | {np.median(d_):.1f} µs |")
     unc = max(o1["min_rtt_ns"], o2["min_rtt_ns"]) / 2e3
     drift = abs(o1["offset_ns"] - o2["offset_ns"]) / 1e3
     print("\n".join(lines))
