@@ -1239,11 +1239,17 @@ def gpu_arm(args):
     }
     # ---- cold-read floor of the in-situ restores (same bytes per warp, same grid, no replay) ----
     # (ctxb_restore_floor: a plain read of the same layout, device-stamped like the resume time)
+    # The resume reads the payload and, for the replay, the re-executed loads'
+    # operands (C2: 16 fragment loads = 2 KiB per warp, cold too); the floor is
+    # a plain read of both (payload-only floor reported beside it).
     floor = {}
+    rx = {"ctxback": pr.site_info(0)["reexec_load_bytes_per_warp"], "full_hw": 0}
     for k, m in (("ctxback", main), ("full_hw", base.get("full_hw"))):
         if m and m.get("context_bytes_per_tb"):
             bpw = int(m["context_bytes_per_tb"]) // 8
-            floor[k] = {"bytes_per_warp": bpw, "resume_floor_us": cb.ctxb_restore_floor(s, bpw, grid, 256, 9),
+            floor[k] = {"bytes_per_warp": bpw, "reexec_load_bytes_per_warp": rx[k],
+                        "resume_floor_us": cb.ctxb_restore_floor(s, bpw + rx[k], grid, 256, 9),
+                        "payload_only_floor_us": cb.ctxb_restore_floor(s, bpw, grid, 256, 9),
                         "resume_us": m["resume_us_median"]}
             floor[k]["frac_of_floor"] = floor[k]["resume_floor_us"] / max(1e-9, m["resume_us_median"])
     # ---- poll overhead, bulk roofline ----

@@ -255,6 +255,9 @@ typedef struct {
   uint32_t live_bytes_per_warp;    /* the LIVE plan of the same site (fallback)     */
   uint32_t defer_site;             /* CTXB_DEFER: site a preemption arriving here is
                                       carried to (== this site: no deferral)          */
+  uint32_t reexec_load_bytes_per_warp; /* bytes the resume's re-executed loads read per
+                                      warp (128 B vector / 4 B scalar each): memory
+                                      traffic of the replay beside the payload      */
 } ctxb_site_info_t;
 
 typedef struct {

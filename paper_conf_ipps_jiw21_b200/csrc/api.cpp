@@ -780,6 +780,10 @@ int ctxb_site_info(const ctxb_program* p, uint32_t site, ctxb_site_info_t* o) {
   o->payload_bytes_per_warp = pl.payload_bytes;
   o->live_bytes_per_warp = p->an.live[site].payload_bytes;
   o->defer_site = (uint32_t)p->an.defer[site];
+  o->reexec_load_bytes_per_warp = 0;
+  for (const Event& e : pl.schedule)
+    if (e.is_x && p->prog.ins[e.j].op == Op::Ldg)
+      o->reexec_load_bytes_per_warp += p->prog.is_vec(p->prog.ins[e.j].defreg) ? 128u : 4u;
   return CTXB_OK;
 }
 

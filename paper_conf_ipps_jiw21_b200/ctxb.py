@@ -63,7 +63,7 @@ class _Opts(C.Structure):
 class _SiteInfo(C.Structure):
     _fields_ = [(n, C.c_uint32) for n in ("c", "p", "n_vec", "n_scalar", "n_revert_pre", "n_revert_res",
                                           "n_reexec", "payload_bytes_per_warp", "live_bytes_per_warp",
-                                          "defer_site")]
+                                          "defer_site", "reexec_load_bytes_per_warp")]
 
 
 class _ProgInfo(C.Structure):

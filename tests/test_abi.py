@@ -269,3 +269,20 @@ def test_watcher_option_validation():
     a = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | cb.WATCHER, debug=cb.DEBUG_NO_COMPILE)
     b = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
     assert a.source == b.source
+
+
+def test_reexec_load_bytes():
+    """ctxb_site_info_t.reexec_load_bytes_per_warp: C2's window re-executes the
+    next k-step's 8 A and 8 B fragment loads (16 x 128 B, by hand from the IR:
+    the software-pipelined prefetch precedes the poll); Fig 2's main block
+    re-executes only ALU instructions (0 B), its init block its loads."""
+    import json
+    from workloads import configs
+    p = cb.Program(configs.c2(256, 256, 64)["ir"], poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
+    assert p.site_info(0)["reexec_load_bytes_per_warp"] == 16 * 128
+    g = json.load(open(os.path.join(ROOT, "tests", "golden", "fig2.json")))
+    q = cb.Program(g["ir"], debug=cb.DEBUG_NO_COMPILE)
+    s0 = 6                                     # main: after the init block's 5 loads and its branch
+    assert all(q.site_info(k)["reexec_load_bytes_per_warp"] == 0 for k in range(q.num_sites)
+               if q.site_info(k)["c"] >= s0)
+    assert q.site_info(1)["reexec_load_bytes_per_warp"] == 128      # re-executes `ldg v0, inp0[%tid]`
