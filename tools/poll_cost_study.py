@@ -16,6 +16,8 @@ import paper_conf_ipps_jiw21_b200 as cb  # noqa: E402
 from workloads import configs  # noqa: E402
 
 s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
+# SIGNAL=watcher: the preemptions go through CTXB_WATCHER + CTXB_DRAIN_NOTICE (the bench's path)
+SIG = (cb.WATCHER | cb.DRAIN_NOTICE) if os.environ.get("SIGNAL") == "watcher" else 0
 
 
 def timed(prog, grid, bufs, uni=(), reps=7):
@@ -124,7 +126,8 @@ def c4b(trials):
         fl = {"word": 0, "replicas": cb.FLAG_REPLICAS}[fname]
         if True:
             if True:
-                prog = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | fl, load_every=le)
+                prog = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | fl | SIG, load_every=le)
+                grid = prog.persistent_grid()      # room for the watcher warp (a block waiting for it doubles the tail)
                 ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
                 _, _, sizes = bfs(prog, grid, ctx)
                 big = int(np.argmax(sizes))
