@@ -173,8 +173,8 @@ extern "C" {
                              watcher polls that word with system-scope loads and
                              raises the device flag (+ replicas), bypassing the
                              ~7 us stream memory op, which stays as the fallback
-                             on ctrl_stream (env CTXB_HOST_SIGNAL_ONLY=1 drops
-                             it: tests).  A launch that ends unpreempted
+                             on ctrl_stream (ctrl_stream == NULL, or env
+                             CTXB_HOST_SIGNAL_ONLY=1, drops it).  A launch that ends unpreempted
                              releases its watcher when collected.
                              signal_to_drained_us is 0 (the host store is not
                              stream-ordered): use host_us.  Exclusive with

@@ -982,6 +982,7 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
 // the legacy default stream.
 static int check_ctrl(const ctxb_run* r, void* ctrl) {
   if (r->armed) return CTXB_OK;
+  if (r->watching && ctrl == nullptr) return CTXB_OK;   // CTXB_WATCHER alone, no memop fallback
   CUstream cs = (CUstream)ctrl, rs = r->stream;
   if (cs == rs) return fail(CTXB_E_INVALID_ARG, "ctrl_stream must differ from the run's stream");
   if (cs == nullptr || cs == CU_STREAM_LEGACY)
@@ -1025,6 +1026,7 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
   const char* ho = (hf || watch) ? getenv("CTXB_HOST_SIGNAL_ONLY") : nullptr;
   const bool host_only = ho && atoi(ho) != 0;
   CUstream cs = (CUstream)ctrl;
+  const bool no_fallback = (hf || watch) && (host_only || ctrl == nullptr);
   if (r->armed) {
     // CTXB_ARMED_SIGNAL: release the signal enqueued on the library's stream at launch
     *(static_cast<volatile uint32_t*>(r->hflag) + 16) = r->gate_seq;
@@ -1032,9 +1034,10 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     r->armed = false;
     cs = r->arm;
   } else {
-    CU(d.cuEventRecord(r->evf, cs));
-    if (!((hf || watch) && host_only))
+    if (!no_fallback) {
+      CU(d.cuEventRecord(r->evf, cs));
       if (int rc = write_signal(r, cs)) return rc;
+    }
   }
   // env CTXB_PREEMPT_TIMEOUT_US > 0: give up waiting for the drain after that
   // long (a kernel without reachable poll sites); the signal stays raised and
@@ -1064,7 +1067,7 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     r->state = RUN_DRAINED;
     return CTXB_OK;
   }
-  CU(d.cuStreamSynchronize(cs));
+  if (cs) CU(d.cuStreamSynchronize(cs));   // the signal stream (none: watcher without fallback)
   int rc = collect(r);
   if (rc) return rc;
   {
@@ -1091,7 +1094,7 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
     for (auto b : blk) st->blocks_preempted += b;
     st->latency_us = st->warps_preempted ? (double)(tmax - tmin) * 1e-3 : 0.0;
     float ms = 0;
-    CU(d.cuEventElapsedTime(&ms, r->evf, r->ev1));
+    if (!(hf || watch)) CU(d.cuEventElapsedTime(&ms, r->evf, r->ev1));
     // with CTXB_HOST_SIGNAL / CTXB_WATCHER the signal is the host store, which the event does not bound
     st->signal_to_drained_us = (hf || watch) ? 0.0 : (double)ms * 1e3;
   }
@@ -1107,6 +1110,7 @@ int ctxb_preempt_async(ctxb_run* r, void* ctrl) {
     *static_cast<volatile uint32_t*>(r->hflag) = 1u;
     std::atomic_thread_fence(std::memory_order_seq_cst);
   }
+  const bool watched = r->watching;
   if (r->watching) {   // CTXB_WATCHER: the watcher relays the host store (the memop stays as the fallback)
     *(static_cast<volatile uint32_t*>(r->hflag) + 8) = r->gate_seq;
     std::atomic_thread_fence(std::memory_order_seq_cst);
@@ -1116,7 +1120,7 @@ int ctxb_preempt_async(ctxb_run* r, void* ctrl) {
     *(static_cast<volatile uint32_t*>(r->hflag) + 16) = r->gate_seq;
     std::atomic_thread_fence(std::memory_order_seq_cst);
     r->armed = false;
-  } else {
+  } else if (!(watched && ctrl == nullptr)) {
     CU(d.cuEventRecord(r->evf, (CUstream)ctrl));
     if (int rc = write_signal(r, (CUstream)ctrl)) return rc;
   }
