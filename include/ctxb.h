@@ -336,9 +336,11 @@ int ctxb_site_plan_text(const ctxb_program* prog, uint32_t site, int live, char*
 /* The generated CUDA C++ source (same buffer convention). */
 int ctxb_generated_source(const ctxb_program* prog, char* buf, size_t cap, size_t* len);
 /* The compiled sm_100a cubin (ELF) of the program's two kernels (the normal and
- * the resume kernel): *len = its size; copied to `buf` if cap >= *len, else
- * _BUFFER_TOO_SMALL.  _STATE if compiled with CTXB_DEBUG_NO_COMPILE.  Lets a
- * caller inspect the generated code with its own tools (cuobjdump -sass,
+ * the resume kernel) -- the output of the compile-time pass with
+ * its dedicated routines: *len = its size; copied to caller-owned `buf` if
+ * cap >= *len, else _BUFFER_TOO_SMALL.  _STATE if compiled with
+ * CTXB_DEBUG_NO_COMPILE; _INVALID_ARG on NULL prog / len.  Lets a caller
+ * inspect the generated code with its own tools (cuobjdump -sass,
  * --dump-resource-usage) independently of this library. */
 int ctxb_program_cubin(const ctxb_program* prog, void* buf, size_t cap, size_t* len);
 
@@ -351,7 +353,10 @@ int ctxb_occupancy(ctxb_program* prog, uint32_t* blocks_per_sm, uint32_t* num_sm
 /* The largest grid whose blocks are all resident at once ("persistent
  * thread"): blocks_per_sm * num_sms, one block fewer when the program uses
  * CTXB_WATCHER and the watcher warp does not fit next to blocks_per_sm
- * blocks on an SM.  Needs a GPU. */
+ * blocks on an SM (registers of the larger of the two kernels, warps, blocks,
+ * shared memory).  A persistent kernel launched with more blocks still runs
+ * correctly, but its extra block waits for a free slot (a doubled tail).
+ * Needs a GPU (_CUDA otherwise); _INVALID_ARG on NULL arguments. */
 int ctxb_persistent_grid(ctxb_program* prog, uint32_t* grid);
 
 /* Bytes of device memory a context buffer for `grid_blocks` blocks needs:
