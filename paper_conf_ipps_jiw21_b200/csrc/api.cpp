@@ -434,9 +434,13 @@ extern "C" __global__ void ctxb_watcher(const u32* hw, u32 seq, u32* flag, unsig
                                         u32* started, u64* stamp) {
   const u32 lane = threadIdx.x;
   if (lane == 0) asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(started), "r"(seq) : "memory");
+  // The host word only moves forward (31-bit sequence numbers, bit 31 = the
+  // launch ended unpreempted): wait while it is behind seq; raise the flags
+  // only for exactly seq; any later value (a newer launch's) just ends this
+  // watcher, so a stale watcher can never hold the stream.
   u32 v;
   do { asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(hw) : "memory"); }
-  while (v != seq && v != (seq | 0x80000000u));
+  while ((int)(((v & 0x7FFFFFFFu) - seq) << 1) < 0);
   if (v != seq) return;
   for (u32 k = lane; k <= 64u; k += 32u) {
     u32* a = k == 0u ? flag : flag + (rep_off + (u64)(k - 1u) * 4096u) / 4u;
@@ -572,6 +576,7 @@ int launch(ctxb_run* r, bool resume) {
   Driver& d = driver();
   if (r->prog->opt.flags & CTXB_WATCHER) {
     r->gate_seq = (r->gate_seq + 1) & 0x7FFFFFFFu;
+    if (r->gate_seq == 0) r->gate_seq = 1;   // 0 is the host word's initial value
     if (int rc = launch_watcher(r)) return rc;
   }
   CU(d.cuEventRecord(r->ev0, r->stream));
