@@ -1306,7 +1306,9 @@ def gpu_arm(args):
     c5_total = None
     if "c5" in extra_cfg:
         c5_total = allsum(ws, extra_cfg["c5"]["modes"]["ctxback"]["batch_jobs_per_s_with_trace"])
-    launches = int(sum(r["launches"] for r in recs))
+    # libctxb kernels in the timed steps: each launch / resume of the victim, and
+    # with CTXB_WATCHER its watcher warp's kernel
+    launches = int(sum(r["launches"] for r in recs)) * (2 if SIGNAL_FLAGS & cb.WATCHER else 1)
     if rank != 0:
         return None
     cpu = None
