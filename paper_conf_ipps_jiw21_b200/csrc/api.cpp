@@ -139,11 +139,19 @@ struct ctxb_run {
   uint32_t drain_base = 0, drain_total = 0;   // exit count before this launch; after it
   // CTXB_ARMED_SIGNAL: release a pending armed signal of a launch that was not
   // preempted and clear the flag it raises (off the preemption path).
+  // CTXB_WATCHER: the launch will not be preempted any more (the caller waits
+  // for its end, or it ended) -> the watcher exits without raising the flag.
+  // Done *before* waiting for the victim: under tools that serialise kernels
+  // (compute-sanitizer, ncu) the victim only starts once the watcher ends.
+  void release_watcher() {
+    if (!watching) return;
+    watching = false;
+    *(static_cast<volatile uint32_t*>(hflag) + 8) = gate_seq | 0x80000000u;
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+  }
   void disarm() {
-    if (watching) {   // CTXB_WATCHER: the launch ended unpreempted -> the watcher exits
-      watching = false;
-      *(static_cast<volatile uint32_t*>(hflag) + 8) = gate_seq | 0x80000000u;
-      std::atomic_thread_fence(std::memory_order_seq_cst);
+    if (watching) {   // the launch ended unpreempted
+      release_watcher();
       driver().cuStreamSynchronize(arm);
     }
     if (!armed) return;
@@ -161,6 +169,7 @@ struct ctxb_run {
       if (flag) {   // return the resources to the program's pool
         // a launch still running keeps its flag / stamps: let it finish first
         // (disarming would otherwise preempt it)
+        release_watcher();
         if (state == RUN_RUNNING) driver().cuStreamSynchronize(stream);
         disarm();
         prog->pool.push_back({flag, stamps, forced, n_warps, ev0, ev1, evf, hflag, hflag_dev, arm, gate_seq,
@@ -1170,6 +1179,7 @@ int ctxb_wait(ctxb_run* r, int* finished) {
   if (!r) return fail(CTXB_E_INVALID_ARG, "NULL run");
   if (int rc = settle(r)) return rc;
   if (r->state == RUN_RUNNING) {
+    r->release_watcher();
     CU(driver().cuStreamSynchronize(r->stream));
     int rc = collect(r);
     if (rc) return rc;
