@@ -178,7 +178,10 @@ extern "C" {
                              releases its watcher when collected.
                              signal_to_drained_us is 0 (the host store is not
                              stream-ordered): use host_us.  Exclusive with
-                             CTXB_ARMED_SIGNAL (_INVALID_ARG)                  */
+                             CTXB_ARMED_SIGNAL (_INVALID_ARG).  No watcher is
+                             started under Nsight Compute or with env
+                             CTXB_NO_WATCHER=1 (the memop is then the signal,
+                             on the library's stream if ctrl_stream is NULL)  */
 
 #define CTXB_MODE_CTXBACK 0u /* per site: least-context flashback-point */
 #define CTXB_MODE_LIVE    1u /* save LIVE_IN(site) (ref [4])              */

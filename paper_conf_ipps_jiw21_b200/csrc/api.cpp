@@ -497,6 +497,18 @@ int probe_module(CUcontext c, Probe** out) {
 
 // CTXB_WATCHER: launch the watcher warp of run r's current launch on the
 // library's signal stream and make the victim's stream wait until it runs.
+// Under Nsight Compute every kernel launch is profiled to completion inside
+// the launch call, so a watcher kernel (which ends only when the host tells it
+// to) would never return: no watcher there (ncu sets
+// NV_COMPUTE_PROFILER_PERFWORKS_DIR); CTXB_NO_WATCHER=1 does the same.  The
+// preemption then takes the stream memory op (on ctrl_stream, or on the
+// library's signal stream when ctrl_stream is NULL).
+bool watcher_disabled() {
+  static const bool off = getenv("NV_COMPUTE_PROFILER_PERFWORKS_DIR") != nullptr ||
+                          (getenv("CTXB_NO_WATCHER") && atoi(getenv("CTXB_NO_WATCHER")) != 0);
+  return off;
+}
+
 int launch_watcher(ctxb_run* r) {
   Probe* P = nullptr;
   {
@@ -583,7 +595,7 @@ int launch(ctxb_run* r, bool resume) {
   pack_params(r, r->prog, blob);
   void* args[] = {blob.data()};
   Driver& d = driver();
-  if (r->prog->opt.flags & CTXB_WATCHER) {
+  if ((r->prog->opt.flags & CTXB_WATCHER) && !watcher_disabled()) {
     r->gate_seq = (r->gate_seq + 1) & 0x7FFFFFFFu;
     if (r->gate_seq == 0) r->gate_seq = 1;   // 0 is the host word's initial value
     if (int rc = launch_watcher(r)) return rc;
@@ -996,7 +1008,9 @@ int ctxb_launch(ctxb_program* p, uint32_t grid, void* const* buffers, const uint
 // the legacy default stream.
 static int check_ctrl(const ctxb_run* r, void* ctrl) {
   if (r->armed) return CTXB_OK;
-  if (r->watching && ctrl == nullptr) return CTXB_OK;   // CTXB_WATCHER alone, no memop fallback
+  // CTXB_WATCHER with ctrl == NULL: the watcher alone (or, where no watcher
+  // runs, the memop on the library's own non-blocking signal stream)
+  if ((r->prog->opt.flags & CTXB_WATCHER) && ctrl == nullptr) return CTXB_OK;
   CUstream cs = (CUstream)ctrl, rs = r->stream;
   if (cs == rs) return fail(CTXB_E_INVALID_ARG, "ctrl_stream must differ from the run's stream");
   if (cs == nullptr || cs == CU_STREAM_LEGACY)
@@ -1041,6 +1055,7 @@ int ctxb_preempt(ctxb_run* r, void* ctrl, ctxb_preempt_stats* st) {
   const bool host_only = ho && atoi(ho) != 0;
   CUstream cs = (CUstream)ctrl;
   const bool no_fallback = (hf || watch) && (host_only || ctrl == nullptr);
+  if (!watch && !cs && (r->prog->opt.flags & CTXB_WATCHER)) cs = r->arm;   // no watcher ran (profiler)
   if (r->armed) {
     // CTXB_ARMED_SIGNAL: release the signal enqueued on the library's stream at launch
     *(static_cast<volatile uint32_t*>(r->hflag) + 16) = r->gate_seq;
@@ -1135,8 +1150,9 @@ int ctxb_preempt_async(ctxb_run* r, void* ctrl) {
     std::atomic_thread_fence(std::memory_order_seq_cst);
     r->armed = false;
   } else if (!(watched && ctrl == nullptr)) {
-    CU(d.cuEventRecord(r->evf, (CUstream)ctrl));
-    if (int rc = write_signal(r, (CUstream)ctrl)) return rc;
+    CUstream cs = (ctrl == nullptr && (r->prog->opt.flags & CTXB_WATCHER)) ? r->arm : (CUstream)ctrl;
+    CU(d.cuEventRecord(r->evf, cs));
+    if (int rc = write_signal(r, cs)) return rc;
   }
   // the run stays RUNNING: ctxb_wait / ctxb_query see it drain (PREEMPTED or DONE)
   return CTXB_OK;
