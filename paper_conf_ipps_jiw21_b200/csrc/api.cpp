@@ -440,16 +440,25 @@ extern "C" __global__ void ctxb_probe_stamp(u64* out) { if (threadIdx.x == 0) ou
 // value in the master flag and every replica; seq | 0x80000000 (the launch
 // ended unpreempted) makes it exit.
 extern "C" __global__ void ctxb_watcher(const u32* hw, u32 seq, u32* flag, unsigned long long rep_off, u32 sig,
-                                        u32* started, u64* stamp) {
+                                        u32* started, u64* stamp, const u32* exits, u32 exit_base, u32 nblocks) {
   const u32 lane = threadIdx.x;
   if (lane == 0) asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(started), "r"(seq) : "memory");
   // The host word only moves forward (31-bit sequence numbers, bit 31 = the
   // launch ended unpreempted): wait while it is behind seq; raise the flags
   // only for exactly seq; any later value (a newer launch's) just ends this
-  // watcher, so a stale watcher can never hold the stream.
+  // watcher, so a stale watcher can never hold the stream.  The watcher also
+  // ends once every block of its launch has exited (the launch's exit count,
+  // kept in device memory by the victim): an operation that waits for the
+  // device to go idle (a module load, cudaFree) then waits only for the
+  // victim, as it would without a watcher.
   u32 v;
-  do { asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(hw) : "memory"); }
-  while ((int)(((v & 0x7FFFFFFFu) - seq) << 1) < 0);
+  for (;;) {
+    asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(hw) : "memory");
+    if ((int)(((v & 0x7FFFFFFFu) - seq) << 1) >= 0) break;
+    u32 e;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(e) : "l"(exits) : "memory");
+    if (e - exit_base >= nblocks) return;
+  }
   if (v != seq) return;
   for (u32 k = lane; k <= 64u; k += 32u) {
     u32* a = k == 0u ? flag : flag + (rep_off + (u64)(k - 1u) * 4096u) / 4u;
@@ -519,10 +528,10 @@ int launch_watcher(ctxb_run* r) {
   // the watcher's "started" word: in the drain-notice page (its counter is at
   // offset 0), away from the gather words that a resume launch resets
   CUdeviceptr hw = r->hflag_dev + 32, flag = r->flag, started = r->flag + r->rep_off - FLAG_STRIDE + 128,
-              stamp = r->stamps_watch;
-  uint32_t seq = r->gate_seq, sig = r->sig;
+              stamp = r->stamps_watch, exits = r->flag + r->rep_off - FLAG_STRIDE;
+  uint32_t seq = r->gate_seq, sig = r->sig, base = r->drain_base, nblk = r->grid;
   unsigned long long rep = r->rep_off;
-  void* a[] = {&hw, &seq, &flag, &rep, &sig, &started, &stamp};
+  void* a[] = {&hw, &seq, &flag, &rep, &sig, &started, &stamp, &exits, &base, &nblk};
   CU(d.cuLaunchKernel(P->watch, 1, 1, 1, 32, 1, 1, 0, r->arm, a, nullptr));
   CU(d.cuStreamWaitValue32(r->stream, started, seq, CU_STREAM_WAIT_VALUE_GEQ));
   r->watching = true;

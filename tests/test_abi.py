@@ -259,7 +259,9 @@ def test_gather_resume_default_for_atomics():
 
 def test_watcher_option_validation():
     """CTXB_WATCHER and CTXB_ARMED_SIGNAL both use the library's signal stream:
-    exclusive.  The watcher changes no plan and no generated kernel."""
+    exclusive.  The watcher changes no plan; the generated kernels only count
+    their blocks' exits (so the watcher can end with its launch), without the
+    drain notice's host store."""
     from workloads import configs
     txt = configs.c2(128, 128, 64)["ir"]
     with pytest.raises(cb.CtxbError) as e:
@@ -268,7 +270,9 @@ def test_watcher_option_validation():
     assert e.value.code == -1
     a = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | cb.WATCHER, debug=cb.DEBUG_NO_COMPILE)
     b = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
-    assert a.source == b.source
+    assert [a.plan_text(k) for k in range(a.num_sites)] == [b.plan_text(k) for k in range(b.num_sites)]
+    assert "warp_exit(P, lane, &blk_out)" in a.source and "warp_exit(P, lane, &blk_out)" not in b.source
+    assert "#define CTXB_NOTICE_HOST 0" in a.source
 
 
 def test_reexec_load_bytes():

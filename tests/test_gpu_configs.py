@@ -455,3 +455,47 @@ def test_program_destroyed_before_its_run():
     p2 = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT)   # the library is still healthy
     r2 = p2.launch(4, [X, Y], [], ctx)
     assert r2.wait()
+
+
+def test_two_runs_with_watchers_concurrently():
+    """Two programs, each launch with its own watcher warp, running at the
+    same time on two streams (small grids, so both are resident): preempt
+    both through their watchers alone, resume both, outputs bit-exact; then
+    the same without preemption (each wait releases its watcher)."""
+    import time
+    import torch
+    cb = _cb()
+    c3 = configs.c3(2048, 2048, 64, **configs.BENCH_C3)
+    x = to_dev(c3["buffers"]["X"])
+    y = torch.zeros(2048 * 2048, dtype=torch.int32, device="cuda")
+    c2 = configs.c2(1024, 1024, 1024)
+    a, b = to_dev(c2["buffers"]["A"]), to_dev(c2["buffers"]["B"])
+    c = torch.zeros(1024 * 1024, dtype=torch.int32, device="cuda")
+    fl = cb.ALL | cb.WATCHER | cb.DRAIN_NOTICE
+    p3 = cb.Program(c3["ir"], poll_policy=cb.POLL_EXPLICIT, flags=fl)
+    p2 = cb.Program(c2["ir"], poll_policy=cb.POLL_EXPLICIT, flags=fl, min_blocks_per_sm=2)
+    g3, g2 = 32, 16
+    ctx3 = torch.zeros(p3.context_capacity(g3), dtype=torch.uint8, device="cuda")
+    ctx2 = torch.zeros(p2.context_capacity(g2), dtype=torch.uint8, device="cuda")
+    s3, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    r3, r2 = p3.launch(g3, [x, y], [], ctx3, s3), p2.launch(g2, [a, b, c], [], ctx2, s2)
+    assert r3.wait() and r2.wait()
+    ref3, ref2 = y.clone(), c.clone()
+    npre = 0
+    for delay in (20e-6, 200e-6):
+        y.zero_()
+        c.zero_()
+        torch.cuda.synchronize()
+        r3, r2 = p3.launch(g3, [x, y], [], ctx3, s3), p2.launch(g2, [a, b, c], [], ctx2, s2)
+        t0 = time.perf_counter()
+        while time.perf_counter() < t0 + delay:
+            pass
+        st3, st2 = r3.preempt(None), r2.preempt(None)
+        npre += st3["warps_preempted"] + st2["warps_preempted"]
+        for r, s in ((r3, s3), (r2, s2)):
+            while not r.finished:
+                r.resume(s)
+                r.wait()
+        torch.cuda.synchronize()
+        assert torch.equal(y, ref3) and torch.equal(c, ref2)
+    assert npre > 0
