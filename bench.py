@@ -60,9 +60,9 @@ def parse():
     ap.add_argument("--detail", default=os.path.join(ROOT, "gpurun_out", "bench_detail.json"),
                     help="side file for the full result (per-config, C5, baselines); stdout gets a compact line")
     ap.add_argument("--signal", default="watcher", choices=["watcher", "armed", "memop"],
-                    help="preemption signal of the headline modes: watcher = CTXB_WATCHER | CTXB_DRAIN_NOTICE (a "
-                         "co-resident warp relays a host store; the last warp's exit is noticed in host memory, "
-                         "DESIGN.md 8n); armed = CTXB_ARMED_SIGNAL (pre-enqueued memop behind a host gate, 8j); "
+                    help="preemption signal of the headline modes: watcher = CTXB_WATCHER | CTXB_DRAIN_NOTICE | "
+                         "CTXB_SYNC_POLL (a co-resident warp relays a host store, each poll tests the flag it loads, "
+                         "the last warp's exit is noticed in host memory, DESIGN.md 8n); armed = CTXB_ARMED_SIGNAL (pre-enqueued memop behind a host gate, 8j); "
                          "memop = cuStreamWriteValue32 on the control stream")
     return ap.parse_args()
 
@@ -178,7 +178,15 @@ SIGNAL_FLAGS = 0   # set by gpu_arm from --signal (signal_paths)
 
 def signal_paths(cb):
     """--signal name -> program flags of that preemption-signal path."""
-    return {"watcher": cb.WATCHER | cb.DRAIN_NOTICE, "armed": cb.ARMED_SIGNAL, "memop": 0}
+    return {"watcher": cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL, "armed": cb.ARMED_SIGNAL, "memop": 0}
+
+
+def kernel_flags(cb, drop=0):
+    """The signal path's code-generation part (the synchronous flag test and
+    the exit counting of the drain notice): it is in the deployed kernel, so
+    poll overheads are measured with it; the watcher itself is a separate
+    kernel and is left out (it would change the grid, not the poll)."""
+    return SIGNAL_FLAGS & (cb.SYNC_POLL | cb.DRAIN_NOTICE) & ~drop
 C3_ROWS = 8        # C3 stencil rows per loop iteration, one (reverting) poll site per iteration (configs.BENCH_C3)
 
 
@@ -467,14 +475,16 @@ def poll_tuning(cb, config):
     per iteration, the reverting site only) loads the one flag word at every
     visit; C4b's edge-chunk polls (configs.BENCH_C4B_POLLS) go to 64 flag
     replicas."""
+    # C4b polls at every frontier vertex: a synchronous test (an L2 round trip
+    # per site) would cost 3-5 %, so C4b keeps the pipelined test (drop_flags)
     return {"c4a": dict(extra_flags=cb.SYNC_POLL),
-            "c4b": dict(extra_flags=cb.FLAG_REPLICAS)}.get(config, {})
+            "c4b": dict(extra_flags=cb.FLAG_REPLICAS, drop_flags=cb.SYNC_POLL)}.get(config, {})
 
 
-def _progs(cb, ir_text, debug=0, min_blocks=0, extra_flags=0, load_every=1):
+def _progs(cb, ir_text, debug=0, min_blocks=0, extra_flags=0, load_every=1, drop_flags=0):
     """Every mode of a config, on the headline's signal path (--signal)."""
     return {name: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT if "poll" in ir_text else cb.POLL_EVERY_INSTR,
-                             mode=mode, flags=flags | extra_flags | SIGNAL_FLAGS, debug=debug | dbg,
+                             mode=mode, flags=(flags | extra_flags | SIGNAL_FLAGS) & ~drop_flags, debug=debug | dbg,
                              min_blocks_per_sm=min_blocks, load_every=load_every)
             for name, mode, flags, dbg in _modes(ir_text)}
 
@@ -531,7 +541,8 @@ def _flag_trials(progs, grid, make_bufs, uniforms, check, fracs, T_s):
     return out
 
 
-def _poll_overhead(cb, ir_text, grid, make_bufs, uniforms=(), extra_flags=0, min_blocks=0, reps=9, load_every=1):
+def _poll_overhead(cb, ir_text, grid, make_bufs, uniforms=(), extra_flags=0, min_blocks=0, reps=9, load_every=1,
+                   drop_flags=0):
     """Poll-site (+OSRB copy) overhead, the paper's Fig. 10 quantity: the
     uninterrupted CTXBack kernel vs the same generated kernel with the poll
     sites compiled out (CTXB_DEBUG_NO_POLLS), medians of `reps` launches of
@@ -539,7 +550,8 @@ def _poll_overhead(cb, ir_text, grid, make_bufs, uniforms=(), extra_flags=0, min
     import torch
     progs, ctxs, ts = {}, {}, {}
     for name, dbg in (("polls_ms", 0), ("no_polls_ms", cb.DEBUG_NO_POLLS)):
-        progs[name] = cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | extra_flags, debug=dbg,
+        progs[name] = cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT,
+                                 flags=(cb.ALL | extra_flags | kernel_flags(cb)) & ~drop_flags, debug=dbg,
                                  min_blocks_per_sm=min_blocks, load_every=load_every)
     if grid is None:   # the polled kernel's own persistent grid (no watcher: the signal path is not the poll's cost)
         grid = progs["polls_ms"].persistent_grid()
@@ -718,7 +730,8 @@ def bench_c4a(cb, trials, seed):
     fr = np.random.default_rng(seed + 3).uniform(0.05, 0.95, trials)
     res = _flag_trials(progs, grid, make, [], lambda b: bool(torch.equal(hsum(b[2]), want)), fr, T / 1e3)
     res["static"] = _static(progs["ctxback"], 8)
-    g_own = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | poll_tuning(cb, "c4a")["extra_flags"],
+    g_own = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT,
+                       flags=cb.ALL | poll_tuning(cb, "c4a")["extra_flags"] | kernel_flags(cb),
                        ).persistent_grid()   # the polled kernel's own persistent grid
     if g_own > grid:
         dH = torch.zeros(256 * g_own, dtype=torch.int32, device="cuda")
@@ -816,7 +829,8 @@ def bench_c4b(cb, trials, seed):
             lvl += 1
         return tot
     prs = {key: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, debug=dbg,
-                           flags=cb.ALL | poll_tuning(cb, "c4b").get("extra_flags", 0))
+                           flags=cb.ALL | poll_tuning(cb, "c4b").get("extra_flags", 0) |
+                           kernel_flags(cb, poll_tuning(cb, "c4b")["drop_flags"]))
            for key, dbg in (("polls_ms", 0), ("no_polls_ms", cb.DEBUG_NO_POLLS))}
     tv = {key: [] for key in prs}
     g_own = prs["polls_ms"].persistent_grid()   # the polled kernel's own persistent grid (no watcher)
@@ -921,7 +935,8 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
         for k, (txt, mb) in irs.items():
             tune = poll_tuning(cb, k)
             progs[k] = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, mode=mode_id[mode], min_blocks_per_sm=mb,
-                                  flags=cb.ALL | tune.get("extra_flags", 0) | (SIGNAL_FLAGS if mode != "none" else 0),
+                                  flags=(cb.ALL | tune.get("extra_flags", 0) | (SIGNAL_FLAGS if mode != "none" else 0))
+                                  & ~tune.get("drop_flags", 0),
                                   load_every=tune.get("load_every", 1))
             grids[k] = progs[k].persistent_grid()
             ctxs[k] = torch.empty(progs[k].context_capacity(grids[k]), dtype=torch.uint8, device="cuda")

@@ -221,7 +221,8 @@ def test_c2s_full_flag_equals_c2():
                                         ("c2", "notice"), ("c3r2", "notice"), ("c2s", "notice"),
                                         ("c2", "watcher"), ("c3b", "watcher"), ("c4a", "watcher"), ("c2s", "watcher"),
                                         ("c2", "watcher_only"), ("c3b", "watcher_only"), ("c2", "watcher_gather"),
-                                        ("c3b", "watcher_gather"), ("c2", "watcher_noctrl"), ("c4a", "watcher_noctrl")])
+                                        ("c3b", "watcher_gather"), ("c2", "watcher_noctrl"), ("c4a", "watcher_noctrl"),
+                                        ("c2", "watcher_sync"), ("c3b", "watcher_sync"), ("c2s", "watcher_sync")])
 def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
     """random flag times, repeated and nested
     preempt -> resume -> preempt ... cycles (each resume can be preempted
@@ -265,11 +266,12 @@ def test_flag_mode_repeated_nested_preemption(which, host, monkeypatch):
              "watcher": cb.WATCHER | cb.DRAIN_NOTICE, "watcher_only": cb.WATCHER,
              "watcher_gather": cb.WATCHER | cb.DRAIN_NOTICE | cb.GATHER_RESUME,
              "watcher_noctrl": cb.WATCHER | cb.DRAIN_NOTICE,
+             "watcher_sync": cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL,   # the bench's signal path
              "replicas+load4": cb.FLAG_REPLICAS, True: cb.HOST_SIGNAL, False: 0}[host]
     prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=mb, flags=cb.ALL | extra,
                       load_every=4 if host in ("load4", "replicas+load4", "combo") else 1)
     grid = prog.persistent_grid()
-    if host in ("watcher", "watcher_only", "watcher_gather", "watcher_noctrl") and which in ("c2", "c2s"):
+    if host in ("watcher", "watcher_only", "watcher_gather", "watcher_noctrl", "watcher_sync") and which in ("c2", "c2s"):
         bps, nsm = prog.occupancy()
         assert grid == bps * nsm - 1      # the full register file leaves no room for the watcher warp
     if bufs[out_i] is None:

@@ -118,12 +118,15 @@ def c4b(trials):
     ctx = torch.empty(base.context_capacity(grid), dtype=torch.uint8, device="cuda")
     bfs(base, grid, ctx)
     t0 = float(np.median([bfs(base, grid, ctx)[0] for _ in range(5)]))
-    variants = [(p, f, le) for p in ("both", "vertex", "edge") for f in ("word", "replicas") for le in (1, 4)]
+    variants = [(p, f, str(le)) for p in ("both", "vertex", "edge") for f in ("word", "replicas") for le in (1, 4)]
     if os.environ.get("C4B_VARIANTS"):      # e.g. "edge:replicas:1,edge:replicas:2"
-        variants = [(a, b, int(c)) for a, b, c in (v.split(":") for v in os.environ["C4B_VARIANTS"].split(","))]
-    for polls, fname, le in variants:
+        variants = [tuple(v.split(":")) for v in os.environ["C4B_VARIANTS"].split(",")]   # polls:flag:K[:sync]
+    for var in variants:
+        polls, fname, le = var[0], var[1], int(var[2])
         txt = configs.c4b_ir(polls)
-        fl = {"word": 0, "replicas": cb.FLAG_REPLICAS}[fname]
+        fl = {"word": 0, "replicas": cb.FLAG_REPLICAS}[fname] | (cb.SYNC_POLL if len(var) > 3 else 0)
+        if len(var) > 3:
+            fname += " sync"
         if True:
             if True:
                 prog = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | fl | SIG, load_every=le)

@@ -39,6 +39,9 @@ MODES = (("memop", 0, None, None), ("armed", cb.ARMED_SIGNAL, None, None),
          ("watcher", cb.WATCHER, None, None), ("watcher only", cb.WATCHER, None, "1"),
          ("watcher + drain notice", cb.WATCHER | cb.DRAIN_NOTICE, None, None),
          ("armed + drain notice", cb.ARMED_SIGNAL | cb.DRAIN_NOTICE, None, None))
+if os.environ.get("MODES") == "sync":      # the synchronous flag test on the headline path
+    MODES = (("watcher + drain notice", cb.WATCHER | cb.DRAIN_NOTICE, None, None),
+             ("watcher + drain notice + sync poll", cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL, None, None))
 
 
 def main():
