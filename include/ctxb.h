@@ -151,8 +151,10 @@ extern "C" {
                              signal forwards it to every replica; replica
                              pollers read the master at every 64th load (so
                              finished master pollers cannot hide a signal).
-                             Detection takes up to one more poll interval.  For kernels
-                             with frequent polls (C3: 0.90 -> 0.24 ms)       */
+                             Detection takes up to one more poll interval
+                             (none with CTXB_WATCHER, which raises the master
+                             and every replica itself).  For kernels with
+                             frequent polls (C3: 0.90 -> 0.24 ms)            */
 #define CTXB_DRAIN_NOTICE 16384u /* codegen + runtime: the launch's last warp to
                              exit writes its signal value to a word in mapped
                              pinned host memory (one shared-memory count per
@@ -161,7 +163,8 @@ extern "C" {
                              instead of the kernel's completion event: host
                              latency -5 µs on C2, but the kernel's completion
                              (the sysmem write is flushed at kernel end) comes
-                             ~2 µs later                      */
+                             ~2 µs later.  The per-block exit
+                             count alone is also kept for CTXB_WATCHER       */
 
 #define CTXB_WATCHER 32768u /* runtime: every launch (and resume) first starts a
                              one-warp watcher kernel on a library-owned
