@@ -99,20 +99,29 @@ def test_c2_small_forced_nested(mode):
     check_mode(cfg["ir"], 1, cfg["buffers"], scheds, MODES[mode], policy="EXPLICIT", min_blocks=cfg["min_blocks"])
 
 
-@pytest.mark.parametrize("mode", list(MODES))
+@pytest.mark.parametrize("mode", list(MODES) + ["ctxback_prune"])
 def test_c2_full_size_flag(mode):
     """4096^3 on the persistent grid; flag at 30 % and 60 % of T: C bit-exact
     with the uninterrupted run, every preempted warp's header bytes = the
-    mode's plan bytes (FULL_HW: 128 x NUM_REGS)."""
+    mode's plan bytes (FULL_HW: 128 x NUM_REGS); also CTXBack with the
+    demand-driven restore (CTXB_PRUNE, its own plans)."""
     import time
     import torch
     cb = _cb()
     cfg = configs.c2()
     M, N = cfg["M"], cfg["N"]
     op = ir.parse(cfg["ir"])
-    m = MODES[mode]
-    an = A.analyze(op, policy="EXPLICIT", mode=min(m, 2))
-    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, mode=m, min_blocks_per_sm=cfg["min_blocks"])
+    # the NEXT-N4 plan variants run here too (CTXBack mode, their own plans)
+    m = MODES.get(mode, 0)
+    # (CTXB_EXACT is GPU-tested on small kernels: the oracle's exhaustive
+    # search stops at 18 candidate values, C2's windows have more)
+    extra = {"ctxback_prune": (A.FLAG_PRUNE, cb.PRUNE)}.get(mode, (0, 0))
+    an = A.analyze(op, policy="EXPLICIT", mode=min(m, 2), flags=A.FLAGS_ALL | extra[0])
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, mode=m, min_blocks_per_sm=cfg["min_blocks"],
+                      flags=cb.ALL | extra[1])
+    for k, c in enumerate(an.sites):
+        if m == 0:
+            assert prog.plan_text(k) == A.plan_text(op, an.plans[c])
     bps, nsm = prog.occupancy()
     grid = bps * nsm
     dA, dB = to_dev(cfg["buffers"]["A"]), to_dev(cfg["buffers"]["B"])
