@@ -101,7 +101,7 @@ def test_random_programs(seed):
     check(txt, grid, bufs, scheds)
 
 
-@pytest.mark.parametrize("name", ["fig2", "fig3", "fig4", "fig5", "fig6", "r9"])
+@pytest.mark.parametrize("name", ["fig2", "fig3", "fig4", "fig5", "fig6", "r9", "r3", "r3bar", "osrb_select", "n3"])
 def test_paper_figures_on_gpu(name):
     import json
     import os

@@ -83,3 +83,28 @@ def test_defer_targets_by_hand(mode):
     got = [prog.site_info(k)["defer_site"] for k in range(prog.num_sites)]
     want = d["targets_init"] + [t + len(d["targets_init"]) for t in d[f"targets_{mode}_main"]]
     assert got == want
+
+
+def test_osrb_selection_by_hand():
+    """R-7 on tests/golden/osrb_select.json: which irreversible
+    scalar defs are candidates, which one is selected (the one whose backup
+    lets a live result re-execute), and the plans with OSRB on / off at one
+    site -- oracle and C++ analyzer against the hand values."""
+    g, op = load("osrb_select")
+    s0 = op.bbs[op.labels["main"]][0]
+    assert [m - s0 for m in A.osrb_candidates(op)] == g["candidates"]
+    an = A.analyze(op)
+    assert [m - s0 for m in an.backups] == g["selected"]
+    prog = cb.Program(g["ir"], debug=cb.DEBUG_NO_COMPILE)
+    assert [m - s0 for m in prog.backups] == g["selected"]
+    c = s0 + g["site"]
+    assert (an.plans[c].p - s0, an.plans[c].payload_bytes) == tuple(g["osrb_on"])
+    off = A.analyze(op, flags=A.FLAG_RELAXED | A.FLAG_REVERT)
+    assert (off.plans[c].p - s0, off.plans[c].payload_bytes) == tuple(g["osrb_off"])
+    poff = cb.Program(g["ir"], flags=cb.RELAXED | cb.REVERT, debug=cb.DEBUG_NO_COMPILE)
+    k = an.sites.index(c)
+    assert (poff.site_info(k)["p"] - s0, poff.site_info(k)["payload_bytes_per_warp"]) == tuple(g["osrb_off"])
+    for lk, want in g["bytes_osrb_on_main"].items():
+        cc = s0 + int(lk)
+        assert an.plans[cc].payload_bytes == want
+        assert prog.site_info(an.sites.index(cc))["payload_bytes_per_warp"] == want
