@@ -501,3 +501,80 @@ def test_two_runs_with_watchers_concurrently():
         torch.cuda.synchronize()
         assert torch.equal(y, ref3) and torch.equal(c, ref2)
     assert npre > 0
+
+
+@pytest.mark.parametrize("which,path", [("c3", "watcher"), ("c2", "watcher"), ("c3", "armed")])
+def test_watcher_lifecycle_fuzz(which, path):
+    """Seeded random sequences of the run API on the watcher path (C3, C2) and
+    the armed path (C3):
+    preempt with and without stats, preempt_async, blocking waits on
+    unpreempted launches, query polling, resumes, and runs dropped while
+    still running; every job's output bit-exact and nothing hangs (a
+    watchdog aborts the process instead of letting a deadlock sit)."""
+    import faulthandler
+    import sys
+    import time
+    import torch
+    cb = _cb()
+    faulthandler.dump_traceback_later(240, exit=True, file=sys.stderr)
+    try:
+        fl = cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL if path == "watcher" else cb.ARMED_SIGNAL
+        if which == "c3":
+            cfg = configs.c3(**configs.BENCH_C3)
+            ins = [to_dev(cfg["buffers"]["X"])]
+            y = torch.zeros(cfg["W"] * cfg["H"], dtype=torch.int32, device="cuda")
+            mb = 0
+        else:
+            cfg = configs.c2()
+            ins = [to_dev(cfg["buffers"]["A"]), to_dev(cfg["buffers"]["B"])]
+            y = torch.zeros(cfg["M"] * cfg["N"], dtype=torch.int32, device="cuda")
+            mb = 2
+        prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | fl, min_blocks_per_sm=mb)
+        grid = prog.persistent_grid()
+        ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+        s, ctrl = torch.cuda.Stream(), torch.cuda.Stream()
+        bufs = ins + [y]
+        run = prog.launch(grid, bufs, [], ctx, s)
+        assert run.wait()
+        T = run.launch_ms() / 1e3
+        ref = y.clone()
+        import os
+        rng = np.random.default_rng(int(os.environ.get("CTXB_FUZZ_SEED", "2024")))
+        npre = 0
+        for job in range(int(os.environ.get("CTXB_FUZZ_JOBS", "40"))):
+            y.zero_()
+            torch.cuda.synchronize()
+            run = prog.launch(grid, bufs, [], ctx, s)
+            op = int(rng.integers(6))
+            t0 = time.perf_counter()
+            while time.perf_counter() < t0 + rng.uniform(0.0, 0.9) * T:
+                pass
+            if op == 5:                       # drop the run while it may still run; the destructor waits
+                del run
+                torch.cuda.synchronize()
+                assert torch.equal(y, ref)
+                continue
+            c0 = None if path == "watcher" and rng.integers(2) else ctrl   # armed: ctrl unused
+            if op == 0:
+                st = run.preempt(c0)
+                npre += st["warps_preempted"]
+            elif op == 1:
+                assert run.preempt(c0, stats=False) is None
+            elif op == 2:
+                run.preempt_async(c0)
+            elif op == 3:
+                while run.running():
+                    pass
+            # op 4: no preemption, a blocking wait
+            while not run.wait():
+                if rng.integers(3) == 0:      # preempt the resumed launch again at once
+                    run.resume(s)
+                    st = run.preempt(ctrl)
+                    npre += st["warps_preempted"]
+                    continue
+                run.resume(s)
+            torch.cuda.synchronize()
+            assert torch.equal(y, ref), f"job {job} (op {op}) differs"
+        assert npre > 0
+    finally:
+        faulthandler.cancel_dump_traceback_later()
