@@ -503,7 +503,7 @@ def test_two_runs_with_watchers_concurrently():
     assert npre > 0
 
 
-@pytest.mark.parametrize("which,path", [("c3", "watcher"), ("c2", "watcher"), ("c3", "armed")])
+@pytest.mark.parametrize("which,path", [("c3", "watcher"), ("c2", "watcher"), ("c3", "armed"), ("c3", "memop")])
 def test_watcher_lifecycle_fuzz(which, path):
     """Seeded random sequences of the run API on the watcher path (C3, C2) and
     the armed path (C3):
@@ -518,7 +518,7 @@ def test_watcher_lifecycle_fuzz(which, path):
     cb = _cb()
     faulthandler.dump_traceback_later(240, exit=True, file=sys.stderr)
     try:
-        fl = cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL if path == "watcher" else cb.ARMED_SIGNAL
+        fl = {"watcher": cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL, "armed": cb.ARMED_SIGNAL, "memop": 0}[path]
         if which == "c3":
             cfg = configs.c3(**configs.BENCH_C3)
             ins = [to_dev(cfg["buffers"]["X"])]
