@@ -29,6 +29,9 @@ def main():
     h = torch.zeros(256 * 4096, dtype=torch.int32, device="cuda")
     cases = [("c2", c2["ir"], lambda: [a, b, c], 2, 0), ("c2s", configs.c2s()["ir"], lambda: [a, b, c], 2, 0),
              ("c3", c3["ir"], lambda: [x, y], 0, 0), ("c4a", c4["ir"], lambda: [k, st, h.zero_()], 0, 0)]
+    if os.environ.get("C4A_MID"):       # only C4a, with extra sites inside the atomics
+        cases = [(f"c4a_m{m}", configs.c4a_ir(1 << 28, 8, m), lambda: [k, st, h.zero_()], 0, 0)
+                 for m in (0, 1, 3)]
     print("| config | flag test | polled ms | no-polls ms | overhead |")
     print("|---|---|---|---|---|")
     for name, txt, mk, mb, ex in cases:

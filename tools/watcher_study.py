@@ -20,8 +20,8 @@ from workloads import configs  # noqa: E402
 
 
 def setup(which):
-    if which == "c4a":
-        cfg = configs.c4a(1 << 28, grid=1)
+    if which.startswith("c4a"):          # c4a, c4a_m1, c4a_m3: extra poll sites inside the atomics
+        cfg = configs.c4a(1 << 28, grid=1, mid_polls=int(which[5:]) if "_m" in which else 0)
         k = torch.from_numpy(cfg["buffers"]["keys"].view(np.int32)).cuda()
         st = torch.from_numpy(cfg["buffers"]["starts"].view(np.int32)).cuda()
         return cfg["ir"], lambda g: [k, st, torch.zeros(256 * g, dtype=torch.int32, device="cuda")], 0, cb.SYNC_POLL
@@ -39,6 +39,8 @@ MODES = (("memop", 0, None, None), ("armed", cb.ARMED_SIGNAL, None, None),
          ("watcher", cb.WATCHER, None, None), ("watcher only", cb.WATCHER, None, "1"),
          ("watcher + drain notice", cb.WATCHER | cb.DRAIN_NOTICE, None, None),
          ("armed + drain notice", cb.ARMED_SIGNAL | cb.DRAIN_NOTICE, None, None))
+if os.environ.get("MODES") == "headline":    # the bench's signal path only
+    MODES = (("watcher + drain notice + sync poll", cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL, None, None),)
 if os.environ.get("MODES") == "sync":      # the synchronous flag test on the headline path
     MODES = (("watcher + drain notice", cb.WATCHER | cb.DRAIN_NOTICE, None, None),
              ("watcher + drain notice + sync poll", cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL, None, None))
@@ -66,7 +68,7 @@ def main():
             ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
             ts = []
             for _ in range(5):
-                if which == "c4a":
+                if which.startswith("c4a"):
                     bufs[-1].zero_()
                 run = prog.launch(grid, bufs, [], ctx, s)
                 run.wait()
@@ -76,7 +78,7 @@ def main():
             ref = bufs[-1].clone()
             host, lat, spread, s2d, npre = [], [], [], [], 0
             for fr in np.random.default_rng(3).uniform(0.1, 0.9, trials):
-                if which == "c4a":
+                if which.startswith("c4a"):
                     bufs[-1].zero_()
                 run = prog.launch(grid, bufs, [], ctx, s)
                 t0 = time.perf_counter()

@@ -316,7 +316,7 @@ def c3_numpy_reference(x_bits, W, H):
 
 # configs[3]: "histogram + BFS-frontier IR kernels with scalar-operand-limited
 # re-execution (exercises on-chip scalar backup)".
-def c4a_ir(nkeys=1 << 28, per_lane=8):
+def c4a_ir(nkeys=1 << 28, per_lane=8, mid_polls=0):
     """256-bin histogram of u32 keys (bin = key >> 24) with global atomics
     into a per-block private copy of the bins (hist[ctaid*256 + bin]; the
     copies are summed afterwards) so that atomics on the same address only
@@ -354,6 +354,10 @@ def c4a_ir(nkeys=1 << 28, per_lane=8):
     e("  ldg s3, starts[s4]")                         # next base: irreversible scalar overwrite
     e("  poll")
     for j in range(per_lane):
+        # mid_polls > 0: more sites inside the atomics (each after per_lane /
+        # (mid_polls + 1) of them), for a shorter poll interval
+        if mid_polls and j and j % (per_lane // (mid_polls + 1)) == 0:
+            e("  poll")
         e(f"  atom.add _, hist[v{1 + per_lane + j}], 1")
     e("  brnz s2, loop")
     e("done:")
@@ -361,7 +365,7 @@ def c4a_ir(nkeys=1 << 28, per_lane=8):
     return "\n".join(L) + "\n"
 
 
-def c4a(nkeys=1 << 28, skewed=False, per_lane=8, grid=2):
+def c4a(nkeys=1 << 28, skewed=False, per_lane=8, grid=2, mid_polls=0):
     """`grid` = number of blocks the kernel is launched with (the hist buffer
     holds one 256-bin copy per block)."""
     chunk = 32 * per_lane
@@ -374,7 +378,7 @@ def c4a(nkeys=1 << 28, skewed=False, per_lane=8, grid=2):
         keys = r.integers(0, 1 << 32, nkeys, dtype=np.uint64).astype(np.uint32)
     starts = (np.arange(nkeys // chunk, dtype=np.uint64) * chunk).astype(np.uint32)
     bufs = {"keys": keys, "starts": starts, "hist": np.zeros(256 * grid, dtype=np.uint32)}
-    return dict(name="C4a", ir=c4a_ir(nkeys, per_lane), grid=grid, buffers=bufs, uniforms={},
+    return dict(name="C4a", ir=c4a_ir(nkeys, per_lane, mid_polls), grid=grid, buffers=bufs, uniforms={},
                 policy="EXPLICIT", nkeys=nkeys, min_blocks=0)
 
 
