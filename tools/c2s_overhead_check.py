@@ -1,3 +1,6 @@
+"""C2s poll overhead at several grid sizes (polled vs no-polls build,
+interleaved): the 292-295-block anomaly of profiles/r02_poll_placement.md.
+python tools/c2s_overhead_check.py 296,295,288"""
 import sys, numpy as np, torch
 sys.path.insert(0, '/root/repo')
 import bench, paper_conf_ipps_jiw21_b200 as cb

@@ -1,3 +1,6 @@
+"""C4b detection with the memop vs the watcher signal (largest level, 4
+preemptions each): routines span, first-seen -> median / p99 / last-seen
+spread, host latency, watcher raise -> first warp (profiles/r02_poll_placement.md)."""
 import sys, time, numpy as np, torch
 sys.path.insert(0, '/root/repo')
 import paper_conf_ipps_jiw21_b200 as cb

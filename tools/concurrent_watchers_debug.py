@@ -1,3 +1,6 @@
+"""Two watched runs (C3, C2) in flight at once, step by step with a
+faulthandler watchdog logging to gpurun_out/conc.log: the reproduction of
+the module-load deadlock fixed in round 2."""
 import faulthandler, sys, time, os
 sys.path.insert(0, '/root/repo'); sys.path.insert(0, '/root/repo/tests')
 log = open('/root/repo/gpurun_out/conc.log', 'w', buffering=1)
