@@ -213,6 +213,11 @@ extern "C" {
 #define CTXB_DEBUG_NO_FP_SHARE 256u /* keep only the exact sharing of byte-identical
                                     preemption routines: no per-flashback-point
                                     routine with entry offsets (A/B)    */
+#define CTXB_DEBUG_NO_SPEC_RESTORE 512u /* no speculative restore loads: the
+                                    resume kernel issues the payload loads only
+                                    after the header's dispatch (A/B; by default
+                                    up to 16 registers of payload common to every
+                                    site's layout are loaded with the header)   */
 #define CTXB_DEBUG_FENCE_STAMPS 32u /* __threadfence before the t_saved stamp, so
                                     it marks the payload as visible (slower
                                     drain; by default the kernel boundary orders

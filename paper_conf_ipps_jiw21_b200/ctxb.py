@@ -16,7 +16,7 @@ __all__ = [
     "LIB_PATH", "CtxbError", "lib",
     "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "GATHER_RESUME", "SYNC_POLL", "HOST_SIGNAL", "ARMED_SIGNAL", "OSRB_SMEM", "OSRB_LANES", "FLAG_REPLICAS", "DRAIN_NOTICE", "WATCHER", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
-    "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS", "DEBUG_NO_AUTO_GATHER", "DEBUG_NO_FP_SHARE",
+    "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS", "DEBUG_NO_AUTO_GATHER", "DEBUG_NO_FP_SHARE", "DEBUG_NO_SPEC_RESTORE",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "E_TIMEOUT", "EXPORTED_SYMBOLS",
     "ctxb_analyze", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait", "ctxb_context_bytes",
     "ctxb_flag_propagation", "ctxb_restore_floor",
@@ -32,7 +32,7 @@ WATCHER = 32768
 MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
 DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1, 2, 4, 8, 16
-DEBUG_FENCE_STAMPS, DEBUG_NO_AUTO_GATHER, DEBUG_NO_FP_SHARE = 32, 128, 256
+DEBUG_FENCE_STAMPS, DEBUG_NO_AUTO_GATHER, DEBUG_NO_FP_SHARE, DEBUG_NO_SPEC_RESTORE = 32, 128, 256, 512
 STATE_NONE, STATE_PREEMPTED, STATE_DONE = 0, 1, 2
 NEVER = 0xFFFFFFFF
 E_TIMEOUT = -8   # ctxb_preempt gave up waiting (env CTXB_PREEMPT_TIMEOUT_US)

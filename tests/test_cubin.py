@@ -91,3 +91,38 @@ def test_c2_stubs_are_128bit_and_spill_free():
     n_st = sum(1 for n in names if n.startswith("STG") and n.endswith(".128") and ".EF" in n)
     n_ld = sum(1 for n in names if n.startswith("LDG") and n.endswith(".128") and ".EF" in n)
     assert n_st >= 16 and n_ld >= 16, (n_st, n_ld)
+
+
+def _resume_sass_order(prog):
+    """Offsets of the first EXIT and of the evict-first payload loads in ctxb_resume."""
+    sass = _cuobjdump(prog.cubin(), "-sass", "-fun", "ctxb_resume")
+    first_exit, ef_loads = None, []
+    for line in sass.splitlines():
+        m = re.match(r"\s*/\*([0-9a-f]{4,})\*/\s+(@!?P\d\s+)?(\w+)(\.[A-Z0-9.]+)?", line)
+        if not m:
+            continue
+        off, op, mod = int(m.group(1), 16), m.group(3), m.group(4) or ""
+        if op == "EXIT" and first_exit is None:
+            first_exit = off
+        if op == "LDG" and ".EF" in mod:
+            ef_loads.append(off)
+    return first_exit, ef_loads
+
+
+def test_speculative_restore_loads_precede_the_header_test():
+    """C3's whole payload (4 loads, <= 16 registers) is loaded
+    together with the header, before the header test's EXIT; with
+    CTXB_DEBUG_NO_SPEC_RESTORE every payload load follows it."""
+    cb = _cb()
+    ir_ = configs.c3(**configs.BENCH_C3)["ir"]
+    spec = cb.Program(ir_, poll_policy=cb.POLL_EXPLICIT)
+    assert spec.source.count("_spec(pay") == 4 and "sdep" in spec.source
+    ex, lds = _resume_sass_order(spec)
+    assert ex is not None and sum(1 for x in lds if x < ex) == 4, (ex, lds)
+    off = cb.Program(ir_, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_SPEC_RESTORE)
+    assert "_spec(pay" not in off.source
+    ex, lds = _resume_sass_order(off)
+    assert ex is not None and lds and all(x > ex for x in lds), (ex, lds)
+    # C2's plans hold 68-70 values: nothing is speculated (register budget)
+    c2 = cb.Program(configs.c2(256, 256, 64)["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=2)
+    assert "_spec(pay" not in c2.source

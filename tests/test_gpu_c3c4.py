@@ -24,12 +24,12 @@ def _cb():
     return cb
 
 
-def forced_parity(cfg, grid, nsched, max_visit, skip=(), compare=None, seed=5, flags=7, prog_flags=0):
+def forced_parity(cfg, grid, nsched, max_visit, skip=(), compare=None, seed=5, flags=7, prog_flags=0, debug=0):
     cb = _cb()
     op = ir.parse(cfg["ir"])
     an = A.analyze(op, policy="EXPLICIT", flags=flags)
     prog = cb.Program(cfg["ir"], flags=flags | prog_flags, poll_policy=cb.POLL_EXPLICIT,
-                      debug=cb.DEBUG_FORCED | cb.DEBUG_POISON)
+                      debug=cb.DEBUG_FORCED | cb.DEBUG_POISON | debug)
     for k, c in enumerate(an.sites):
         assert prog.plan_text(k) == A.plan_text(op, an.plans[c])
     names = list(op.buffers)
@@ -68,6 +68,13 @@ def test_c3_small_forced_bench_placement():
     cfg = configs.c3(512, 128, 64, **configs.BENCH_C3)
     an = forced_parity(cfg, 4, 3, 16)
     assert len(an.sites) == 1 and an.plans[an.sites[0]].n_revert_res + an.plans[an.sites[0]].n_revert_pre > 0
+
+
+def test_c3_small_forced_no_spec_restore():
+    """The A/B build without speculative restore loads: the
+    bench placement's payload is loaded after the header's dispatch."""
+    cfg = configs.c3(512, 128, 64, **configs.BENCH_C3)
+    forced_parity(cfg, 4, 3, 16, debug=_cb().DEBUG_NO_SPEC_RESTORE)
 
 
 def test_c3_small_forced_rank_resume():
