@@ -32,6 +32,12 @@ def main():
     if os.environ.get("C4A_MID"):       # only C4a, with extra sites inside the atomics
         cases = [(f"c4a_m{m}", configs.c4a_ir(1 << 28, 8, m), lambda: [k, st, h.zero_()], 0, 0)
                  for m in (0, 1, 3)]
+    if os.environ.get("C4A_PL"):        # only C4a, with other chunk sizes (keys per lane)
+        cases = []
+        for p in os.environ["C4A_PL"].split(","):
+            cp = configs.c4a(1 << 28, grid=1, per_lane=int(p))      # its own chunk starts
+            stp = torch.from_numpy(cp["buffers"]["starts"].view(np.int32)).cuda()
+            cases.append((f"c4a_p{p}", cp["ir"], lambda stp=stp: [k, stp, h.zero_()], 0, 0))
     print("| config | flag test | polled ms | no-polls ms | overhead |")
     print("|---|---|---|---|---|")
     for name, txt, mk, mb, ex in cases:

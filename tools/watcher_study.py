@@ -20,8 +20,9 @@ from workloads import configs  # noqa: E402
 
 
 def setup(which):
-    if which.startswith("c4a"):          # c4a, c4a_m1, c4a_m3: extra poll sites inside the atomics
-        cfg = configs.c4a(1 << 28, grid=1, mid_polls=int(which[5:]) if "_m" in which else 0)
+    if which.startswith("c4a"):          # c4a, c4a_m1, c4a_m3: extra poll sites inside the atomics; c4a_p4: 4 keys / lane
+        cfg = configs.c4a(1 << 28, grid=1, mid_polls=int(which[5:]) if "_m" in which else 0,
+                          per_lane=int(which[5:]) if "_p" in which else 8)
         k = torch.from_numpy(cfg["buffers"]["keys"].view(np.int32)).cuda()
         st = torch.from_numpy(cfg["buffers"]["starts"].view(np.int32)).cuda()
         return cfg["ir"], lambda g: [k, st, torch.zeros(256 * g, dtype=torch.int32, device="cuda")], 0, cb.SYNC_POLL
