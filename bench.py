@@ -1496,7 +1496,8 @@ def reference_arm(args):
     timed = samp[args.warmup:]
     v = float(np.median([x["latency_us"] for x in timed]))
     wall = sum(x["wall_s"] for x in timed)
-    return {"impl": "reference", "metric": METRIC, "value": round(v, 3), "unit": "us", "n_gpus": 0,
+    return {"impl": "reference", "metric": METRIC, "value": round(v, 3), "unit": "us",
+            "n_gpus": args.gpus, "device": "cpu (host cores; the oracle runs no GPU work)",
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1e3 * wall / max(1, len(timed)), 3),
             "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic",
