@@ -174,11 +174,20 @@ class Clocks:
 # ---- the GPU arm --------------------------------------------------------------
 
 SIGNAL_FLAGS = 0   # set by gpu_arm from --signal (signal_paths)
+SIGNAL_DEBUG = 0   # CTXB_DEBUG_NO_AUTO_SIGNAL for the non-default signal paths
 
 
 def signal_paths(cb):
-    """--signal name -> program flags of that preemption-signal path."""
+    """--signal name -> program flags of that preemption-signal path.  The
+    watcher path is what ctxb_analyze picks by default for C2 (DESIGN.md 8q;
+    gpu_arm checks it); the bench spells it out and builds every program with
+    CTXB_DEBUG_NO_AUTO_SIGNAL (signal_debug), so each mode gets exactly the
+    flags named here and in poll_tuning."""
     return {"watcher": cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL, "armed": cb.ARMED_SIGNAL, "memop": 0}
+
+
+def no_auto(cb):
+    return cb.DEBUG_NO_AUTO_SIGNAL
 
 
 def kernel_flags(cb, drop=0):
@@ -196,7 +205,7 @@ def make_c2(cb, size, mode, debug=0, flags=None):
     flags=None: CTXB_ALL plus the headline's signal option (--signal)."""
     from workloads import configs
     ir_text = configs.c2_ir(size, size, size, polls="iter")
-    return cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, mode=mode, debug=debug, min_blocks_per_sm=2,
+    return cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, mode=mode, debug=debug | no_auto(cb), min_blocks_per_sm=2,
                       flags=cb.ALL | SIGNAL_FLAGS if flags is None else flags)
 
 
@@ -484,7 +493,8 @@ def poll_tuning(cb, config):
 def _progs(cb, ir_text, debug=0, min_blocks=0, extra_flags=0, load_every=1, drop_flags=0):
     """Every mode of a config, on the headline's signal path (--signal)."""
     return {name: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT if "poll" in ir_text else cb.POLL_EVERY_INSTR,
-                             mode=mode, flags=(flags | extra_flags | SIGNAL_FLAGS) & ~drop_flags, debug=debug | dbg,
+                             mode=mode, flags=(flags | extra_flags | SIGNAL_FLAGS) & ~drop_flags,
+                             debug=debug | dbg | no_auto(cb),
                              min_blocks_per_sm=min_blocks, load_every=load_every)
             for name, mode, flags, dbg in _modes(ir_text)}
 
@@ -551,7 +561,7 @@ def _poll_overhead(cb, ir_text, grid, make_bufs, uniforms=(), extra_flags=0, min
     progs, ctxs, ts = {}, {}, {}
     for name, dbg in (("polls_ms", 0), ("no_polls_ms", cb.DEBUG_NO_POLLS)):
         progs[name] = cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT,
-                                 flags=(cb.ALL | extra_flags | kernel_flags(cb)) & ~drop_flags, debug=dbg,
+                                 flags=(cb.ALL | extra_flags | kernel_flags(cb)) & ~drop_flags, debug=dbg | no_auto(cb),
                                  min_blocks_per_sm=min_blocks, load_every=load_every)
     if grid is None:   # the polled kernel's own persistent grid (no watcher: the signal path is not the poll's cost)
         grid = progs["polls_ms"].persistent_grid()
@@ -732,7 +742,7 @@ def bench_c4a(cb, trials, seed):
     res["static"] = _static(progs["ctxback"], 8)
     g_own = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT,
                        flags=cb.ALL | poll_tuning(cb, "c4a")["extra_flags"] | kernel_flags(cb),
-                       ).persistent_grid()   # the polled kernel's own persistent grid
+                       debug=no_auto(cb)).persistent_grid()   # the polled kernel's own persistent grid
     if g_own > grid:
         dH = torch.zeros(256 * g_own, dtype=torch.int32, device="cuda")
     res["poll_overhead"] = _poll_overhead(cb, cfg["ir"], g_own, make, **poll_tuning(cb, "c4a"))   # incl. the OSRB copy
@@ -828,7 +838,7 @@ def bench_c4b(cb, trials, seed):
             nf = int(cnt.item())
             lvl += 1
         return tot
-    prs = {key: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, debug=dbg,
+    prs = {key: cb.Program(ir_text, poll_policy=cb.POLL_EXPLICIT, debug=dbg | no_auto(cb),
                            flags=cb.ALL | poll_tuning(cb, "c4b").get("extra_flags", 0) |
                            kernel_flags(cb, poll_tuning(cb, "c4b")["drop_flags"]))
            for key, dbg in (("polls_ms", 0), ("no_polls_ms", cb.DEBUG_NO_POLLS))}
@@ -937,7 +947,7 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
             progs[k] = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, mode=mode_id[mode], min_blocks_per_sm=mb,
                                   flags=(cb.ALL | tune.get("extra_flags", 0) | (SIGNAL_FLAGS if mode != "none" else 0))
                                   & ~tune.get("drop_flags", 0),
-                                  load_every=tune.get("load_every", 1))
+                                  load_every=tune.get("load_every", 1), debug=no_auto(cb))
             grids[k] = progs[k].persistent_grid()
             ctxs[k] = torch.empty(progs[k].context_capacity(grids[k]), dtype=torch.uint8, device="cuda")
         dev["H"] = torch.zeros(256 * grids["c4a"], dtype=torch.int32, device="cuda")
@@ -1190,6 +1200,10 @@ def gpu_arm(args):
     cfg = configs.c2(size, size, size)
     M = N = K = size
     progs = {"ctxback": make_c2(cb, size, cb.MODE_CTXBACK)}
+    # is the headline's signal path what ctxb_analyze picks by default?
+    default_flags = cb.Program(configs.c2_ir(size, size, size, polls="iter"), poll_policy=cb.POLL_EXPLICIT,
+                               min_blocks_per_sm=2, debug=cb.DEBUG_NO_COMPILE).info["flags"]
+    signal_is_default = default_flags == progs["ctxback"].info["flags"]
     if not args.no_baselines:
         progs["live"] = make_c2(cb, size, cb.MODE_LIVE)
         progs["full_hw"] = make_c2(cb, size, cb.MODE_FULL_HW)
@@ -1199,7 +1213,7 @@ def gpu_arm(args):
         progs["full_hw_gather"] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | cb.GATHER_RESUME | SIGNAL_FLAGS)
         # the other signal paths next to the headline's
         for oname, other in signal_paths(cb).items():
-            if oname != args.signal:
+            if oname != args.signal:   # make_c2 keeps exactly these flags (CTXB_DEBUG_NO_AUTO_SIGNAL)
                 progs["ctxback_" + oname] = make_c2(cb, size, cb.MODE_CTXBACK, flags=cb.ALL | other)
                 progs["full_hw_" + oname] = make_c2(cb, size, cb.MODE_FULL_HW, flags=cb.ALL | other)
     # one persistent grid for every mode (room for the watcher warp where a mode uses it)
@@ -1389,7 +1403,7 @@ def gpu_arm(args):
             "context_pct": (round(100 * (1 - main["context_bytes_per_tb"] / base["full_hw"]["context_bytes_per_tb"]), 2)
                             if "full_hw" in base and base["full_hw"].get("context_bytes_per_tb") and
                             main.get("context_bytes_per_tb") else None)},
-        "signal": args.signal,
+        "signal": args.signal + ("=default" if signal_is_default else ""),
         "other_signal_reduction": {k: _reduction(base, "ctxback_" + k, "full_hw_" + k)
                                    for k in ("watcher", "armed", "memop") if "ctxback_" + k in base},
         "other_signal_host_latency_us": {k: [base.get("ctxback_" + k, {}).get("host_latency_us_median"),

@@ -218,6 +218,24 @@ extern "C" {
                                     after the header's dispatch (A/B; by default
                                     up to 16 registers of payload common to every
                                     site's layout are loaded with the header)   */
+#define CTXB_DEBUG_NO_AUTO_SIGNAL 1024u /* keep exactly the caller's signal-path
+                                    and poll-test bits.  By default a program
+                                    with flag-mode poll sites (not _FORCED, not
+                                    _NO_POLLS) gets:
+                                    * CTXB_WATCHER | CTXB_DRAIN_NOTICE unless the
+                                      caller chose a signal path (CTXB_WATCHER,
+                                      CTXB_ARMED_SIGNAL or CTXB_HOST_SIGNAL);
+                                    * the poll test from a cost model, unless the
+                                      caller chose one (CTXB_SYNC_POLL,
+                                      CTXB_FLAG_REPLICAS, flag_depth > 1 or
+                                      load_every > 1): a site on a loop of fewer
+                                      than CTXB_DENSE_POLL_INSTRS IR instructions
+                                      -> CTXB_FLAG_REPLICAS with the pipelined
+                                      test (a synchronous test would add an L2
+                                      round trip to every short iteration);
+                                      otherwise CTXB_SYNC_POLL.
+                                    ctxb_program_info_t.flags reports the result */
+#define CTXB_DENSE_POLL_INSTRS 32u
 #define CTXB_DEBUG_FENCE_STAMPS 32u /* __threadfence before the t_saved stamp, so
                                     it marks the payload as visible (slower
                                     drain; by default the kernel boundary orders
@@ -302,6 +320,13 @@ typedef struct {
   uint32_t n_fp_shared;                /* sites whose preemption routine is their
                                           flashback-point's shared routine, entered at
                                           an offset past the later sites' reverts */
+  uint32_t flags;                      /* the option bits in effect: the caller's plus
+                                          those ctxb_analyze chose by default
+                                          (CTXB_GATHER_RESUME, and the signal path and
+                                          poll test of CTXB_DEBUG_NO_AUTO_SIGNAL)     */
+  uint32_t poll_loop_instrs;           /* IR instructions on the shortest loop through
+                                          a poll site (0 = no site lies on a loop):
+                                          the poll-test cost model's input           */
 } ctxb_program_info_t;
 
 typedef struct {

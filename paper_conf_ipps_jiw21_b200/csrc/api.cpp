@@ -56,6 +56,7 @@ struct ctxb_program {
   std::string src, log;
   std::vector<char> cubin;
   uint32_t num_regs = 0, regs_resume = 0;
+  uint32_t poll_loop = 0;   // IR instructions on the shortest loop through a poll site (0: none)
   uint32_t spill_st = 0, spill_ld = 0, spill_st_res = 0, spill_ld_res = 0;   // ptxas -v bytes
   double t_an = 0, t_cg = 0, t_cc = 0;
   std::mutex mu;
@@ -687,6 +688,52 @@ void free_program(ctxb_program* p) {
   delete p;
 }
 
+// IR instructions on the shortest cycle of the CFG through the basic block of
+// a poll site, over every site (0 = no site lies on a loop): how often a warp
+// meets a poll, the input of the poll-test cost model below.
+static uint32_t shortest_poll_loop(const Program& P, const std::vector<int>& sites) {
+  const size_t nb = P.bbs.size();
+  auto size = [&](size_t b) { return (uint64_t)(P.bbs[b].second - P.bbs[b].first); };
+  std::vector<uint8_t> seen(nb, 0);
+  uint64_t best = UINT64_MAX;
+  for (int c : sites) {
+    if (c < 0 || (size_t)c >= P.bb_of.size()) continue;
+    const size_t b0 = (size_t)P.bb_of[c];
+    if (seen[b0]) continue;
+    seen[b0] = 1;
+    // Dijkstra from b0's successors; the weight of entering a block is its size
+    std::vector<uint64_t> dist(nb, UINT64_MAX);
+    std::vector<uint8_t> done(nb, 0);
+    for (int s2 : P.succ[b0]) dist[s2] = std::min(dist[s2], size(s2));
+    for (;;) {
+      size_t u = nb;
+      for (size_t v = 0; v < nb; v++)
+        if (!done[v] && dist[v] != UINT64_MAX && (u == nb || dist[v] < dist[u])) u = v;
+      if (u == nb || u == b0) break;
+      done[u] = 1;
+      for (int v : P.succ[u]) dist[v] = std::min(dist[v], dist[u] + size(v));
+    }
+    best = std::min(best, dist[b0]);
+  }
+  return best == UINT64_MAX ? 0u : (uint32_t)std::min<uint64_t>(best, UINT32_MAX);
+}
+
+// Default signal path and poll test: the watcher warp relays
+// the host's store to the flag (~2 us instead of the ~7 us stream memory op)
+// and the last warp's drain notice tells the host (P:74 signal, P:54-56
+// drain), unless the caller chose a signal path; a synchronous flag test
+// (detection within one site interval) unless the sites lie on short loops,
+// where one L2 round trip per visit costs several percent and the pipelined
+// test polls one of the flag replicas instead (dense polls of a large grid
+// would queue on one L2 slice).
+static uint32_t default_signal_flags(const Options& o, uint32_t poll_loop) {
+  uint32_t f = 0;
+  if (!(o.flags & (CTXB_WATCHER | CTXB_ARMED_SIGNAL | CTXB_HOST_SIGNAL))) f |= CTXB_WATCHER | CTXB_DRAIN_NOTICE;
+  if (!(o.flags & (CTXB_SYNC_POLL | CTXB_FLAG_REPLICAS)) && o.flag_depth <= 1 && o.load_every <= 1)
+    f |= (poll_loop && poll_loop < CTXB_DENSE_POLL_INSTRS) ? CTXB_FLAG_REPLICAS : CTXB_SYNC_POLL;
+  return f;
+}
+
 extern "C" {
 
 const char* ctxb_last_error(void) { return g_err.c_str(); }
@@ -718,6 +765,9 @@ int ctxb_analyze(const char* ir_text, size_t len, const ctxb_options* opts, ctxb
     for (const Instr& I : p->prog.ins) atomics = atomics || I.op == Op::AtomAdd || I.op == Op::AtomCas;
     if (atomics && !(o.debug & CTXB_DEBUG_NO_AUTO_GATHER)) p->opt.flags |= CTXB_GATHER_RESUME;
     p->an = analyze(p->prog, p->opt);
+    p->poll_loop = shortest_poll_loop(p->prog, p->an.sites);
+    if (!(o.debug & (CTXB_DEBUG_FORCED | CTXB_DEBUG_NO_POLLS | CTXB_DEBUG_NO_AUTO_SIGNAL)) && !p->an.sites.empty())
+      p->opt.flags |= default_signal_flags(p->opt, p->poll_loop);
     double t1 = now_ms();
     p->src = generate_cuda(p->prog, p->an, p->opt, &p->cg);
     double t2 = now_ms();
@@ -783,6 +833,8 @@ int ctxb_program_info(const ctxb_program* p, ctxb_program_info_t* o) {
   o->spill_loads_resume = p->spill_ld_res;
   o->gather_resume = (p->opt.flags & CTXB_GATHER_RESUME) ? 1u : 0u;
   o->n_fp_shared = p->cg.n_fp_shared;
+  o->flags = p->opt.flags;
+  o->poll_loop_instrs = p->poll_loop;
   return CTXB_OK;
 }
 
@@ -1183,7 +1235,15 @@ int ctxb_resume(ctxb_run* r, void* stream, const uint32_t* forced_targets) {
     CU(d.cuOccupancyMaxActiveBlocksPerMultiprocessor(&b, r->mod.resume, r->prog->prog.block, 0));
     CU(d.cuCtxGetDevice(&dev));
     CU(d.cuDeviceGetAttribute(&n, CU_DEVICE_ATTRIBUTE_MULTIPROCESSOR_COUNT, dev));
-    if ((uint64_t)r->grid <= (uint64_t)b * (uint64_t)n) {
+    uint64_t resident = (uint64_t)b * (uint64_t)n;
+    if ((r->prog->opt.flags & CTXB_WATCHER) && !watcher_disabled()) {
+      // the watcher warp takes a slot: a block that cannot be resident beside
+      // it would keep the gathered blocks waiting
+      uint32_t g = 0;
+      if (int rc = ctxb_persistent_grid(r->prog, &g)) return rc;
+      resident = std::min<uint64_t>(resident, g);
+    }
+    if ((uint64_t)r->grid <= resident) {
       // target = blocks with >= 1 preempted warp (one global arrival per block)
       uint32_t nwb = r->prog->prog.block / 32, blocks = 0;
       for (uint32_t b = 0; b < r->grid; b++) {

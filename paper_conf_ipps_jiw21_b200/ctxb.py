@@ -17,6 +17,7 @@ __all__ = [
     "RELAXED", "REVERT", "OSRB", "ALL", "DEFER", "PRUNE", "RANK_RESUME", "EXACT", "GATHER_RESUME", "SYNC_POLL", "HOST_SIGNAL", "ARMED_SIGNAL", "OSRB_SMEM", "OSRB_LANES", "FLAG_REPLICAS", "DRAIN_NOTICE", "WATCHER", "MODE_CTXBACK", "MODE_LIVE", "MODE_FULL", "MODE_FULL_HW",
     "POLL_EVERY_INSTR", "POLL_EVERY_N", "POLL_EXPLICIT",
     "DEBUG_FORCED", "DEBUG_POISON", "DEBUG_NO_POLLS", "DEBUG_NO_COMPILE", "DEBUG_NO_SHARE", "DEBUG_FENCE_STAMPS", "DEBUG_NO_AUTO_GATHER", "DEBUG_NO_FP_SHARE", "DEBUG_NO_SPEC_RESTORE",
+    "DEBUG_NO_AUTO_SIGNAL", "DENSE_POLL_INSTRS",
     "STATE_NONE", "STATE_PREEMPTED", "STATE_DONE", "NEVER", "E_TIMEOUT", "EXPORTED_SYMBOLS",
     "ctxb_analyze", "ctxb_launch", "ctxb_preempt", "ctxb_resume", "ctxb_wait", "ctxb_context_bytes",
     "ctxb_flag_propagation", "ctxb_restore_floor",
@@ -33,6 +34,8 @@ MODE_CTXBACK, MODE_LIVE, MODE_FULL, MODE_FULL_HW = 0, 1, 2, 3
 POLL_EVERY_INSTR, POLL_EVERY_N, POLL_EXPLICIT = 0, 1, 2
 DEBUG_FORCED, DEBUG_POISON, DEBUG_NO_POLLS, DEBUG_NO_COMPILE, DEBUG_NO_SHARE = 1, 2, 4, 8, 16
 DEBUG_FENCE_STAMPS, DEBUG_NO_AUTO_GATHER, DEBUG_NO_FP_SHARE, DEBUG_NO_SPEC_RESTORE = 32, 128, 256, 512
+DEBUG_NO_AUTO_SIGNAL = 1024   # keep the caller's signal-path / poll-test bits (no defaults)
+DENSE_POLL_INSTRS = 32        # sites on a loop shorter than this get the pipelined test + replicas
 STATE_NONE, STATE_PREEMPTED, STATE_DONE = 0, 1, 2
 NEVER = 0xFFFFFFFF
 E_TIMEOUT = -8   # ctxb_preempt gave up waiting (env CTXB_PREEMPT_TIMEOUT_US)
@@ -74,7 +77,7 @@ class _ProgInfo(C.Structure):
                                           "exact_improved", "exact_fallback")] + \
                [("analyze_ms", C.c_double), ("codegen_ms", C.c_double), ("compile_ms", C.c_double)] + \
                [(n, C.c_uint32) for n in ("spill_stores", "spill_loads", "spill_stores_resume", "spill_loads_resume",
-                                          "gather_resume", "n_fp_shared")]
+                                          "gather_resume", "n_fp_shared", "flags", "poll_loop_instrs")]
 
 
 class _PreStats(C.Structure):

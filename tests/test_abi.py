@@ -117,7 +117,8 @@ def test_runtime_options_generate_and_compile():
     (plans identical); both compile for sm_100a with NVRTC."""
     from workloads import configs
     txt = configs.c4a_ir(1 << 14)
-    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE | cb.DEBUG_NO_AUTO_GATHER)
+    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT,
+                      debug=cb.DEBUG_NO_COMPILE | cb.DEBUG_NO_AUTO_GATHER | cb.DEBUG_NO_AUTO_SIGNAL)
     g = cb.Program(txt, flags=cb.ALL | cb.GATHER_RESUME | cb.SYNC_POLL, poll_policy=cb.POLL_EXPLICIT)
     assert g.info["compiled"] == 1
     assert [g.plan_text(k) for k in range(g.num_sites)] == [base.plan_text(k) for k in range(base.num_sites)]
@@ -154,9 +155,9 @@ def test_armed_signal_is_runtime_only():
     kernel source is byte-identical to the default build's."""
     from workloads import configs
     txt = configs.c3()["ir"]
-    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
-    armed = cb.Program(txt, flags=cb.ALL | cb.ARMED_SIGNAL, poll_policy=cb.POLL_EXPLICIT,
-                       debug=cb.DEBUG_NO_COMPILE)
+    dbg = cb.DEBUG_NO_COMPILE | cb.DEBUG_NO_AUTO_SIGNAL   # the memop build, not the default watcher path
+    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=dbg)
+    armed = cb.Program(txt, flags=cb.ALL | cb.ARMED_SIGNAL, poll_policy=cb.POLL_EXPLICIT, debug=dbg)
     assert armed.source == base.source
     with pytest.raises(cb.CtxbError):
         cb.Program(txt, flags=1 << 20, debug=cb.DEBUG_NO_COMPILE)
@@ -214,7 +215,7 @@ def test_flag_replicas_and_load_every_generate():
     load_every (flag loads at every K-th poll visit): plans unchanged, both
     compile for sm_100a; the options reach the generated polls."""
     txt = configs.c3(512, 128, 64)["ir"]
-    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
+    base = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE | cb.DEBUG_NO_AUTO_SIGNAL)
     p = cb.Program(txt, flags=cb.ALL | cb.FLAG_REPLICAS, poll_policy=cb.POLL_EXPLICIT, load_every=4)
     assert p.info["compiled"] == 1
     assert [p.plan_text(k) for k in range(p.num_sites)] == [base.plan_text(k) for k in range(base.num_sites)]
@@ -268,8 +269,9 @@ def test_watcher_option_validation():
         cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | cb.WATCHER | cb.ARMED_SIGNAL,
                    debug=cb.DEBUG_NO_COMPILE)
     assert e.value.code == -1
-    a = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | cb.WATCHER, debug=cb.DEBUG_NO_COMPILE)
-    b = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_NO_COMPILE)
+    dbg = cb.DEBUG_NO_COMPILE | cb.DEBUG_NO_AUTO_SIGNAL
+    a = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | cb.WATCHER, debug=dbg)
+    b = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, debug=dbg)
     assert [a.plan_text(k) for k in range(a.num_sites)] == [b.plan_text(k) for k in range(b.num_sites)]
     assert "warp_exit(P, lane, &blk_out)" in a.source and "warp_exit(P, lane, &blk_out)" not in b.source
     assert "#define CTXB_NOTICE_HOST 0" in a.source

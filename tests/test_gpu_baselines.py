@@ -164,7 +164,9 @@ def test_ctrl_stream_checks():
     import torch
     cb = _cb()
     cfg = configs.c2()
-    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=cfg["min_blocks"])
+    # the stream-memop signal path (the default watcher path accepts ctrl == NULL)
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=cfg["min_blocks"],
+                      debug=cb.DEBUG_NO_AUTO_SIGNAL)
     bps, nsm = prog.occupancy()
     grid = bps * nsm
     dA, dB = to_dev(cfg["buffers"]["A"]), to_dev(cfg["buffers"]["B"])

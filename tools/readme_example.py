@@ -6,9 +6,9 @@ import torch, paper_conf_ipps_jiw21_b200 as cb
 from workloads import configs
 
 cfg = configs.c2()                                         # 4096^3 tiled SGEMM IR kernel
-fast = cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL           # the bench's signal path
-prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=2,
-                  flags=cb.ALL | fast)                       # ctxb_analyze
+prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=2)   # ctxb_analyze
+# defaults: watcher warp + drain notice + synchronous flag test
+assert prog.info["flags"] & (cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL) == cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL
 grid = prog.persistent_grid()                              # every block resident, room for the watcher
 A = torch.from_numpy(cfg["buffers"]["A"].view("int32")).cuda()
 B = torch.from_numpy(cfg["buffers"]["B"].view("int32")).cuda()
