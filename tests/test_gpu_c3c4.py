@@ -240,3 +240,39 @@ def test_c4b_full_flag(replicas, polls):
         nf = int(cnt.item())
         lvl += 1
     assert np.array_equal(from_dev(d_dist), want)
+
+
+@pytest.mark.parametrize("grid_kind", ["persistent", "occupancy"])
+def test_c4a_library_defaults(grid_kind):
+    """The library's defaults on C4a: watcher + drain notice +
+    synchronous test, gathered resume (atomics).  preempt(None) signals through
+    the watcher alone.  On the occupancy grid one block cannot be resident
+    beside the watcher, so the resume must not gather (it would wait for that
+    block); on the persistent grid it gathers.  Bit-exact either way."""
+    import torch
+    cb = _cb()
+    cfg = configs.c4a(1 << 26, grid=1)
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT)
+    want_bits = cb.WATCHER | cb.DRAIN_NOTICE | cb.SYNC_POLL | cb.GATHER_RESUME
+    assert prog.info["flags"] & want_bits == want_bits
+    grid = prog.persistent_grid() if grid_kind == "persistent" else _persistent_grid(prog)
+    keys = cfg["buffers"]["keys"]
+    want = np.bincount(keys >> 24, minlength=256).astype(np.uint32)
+    dK, dS = to_dev(keys), to_dev(cfg["buffers"]["starts"])
+    dH = torch.zeros(256 * grid, dtype=torch.int32, device="cuda")
+    total = lambda: from_dev(dH).reshape(grid, 256).astype(np.uint64).sum(0).astype(np.uint32)  # noqa: E731
+    ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    s = torch.cuda.Stream()
+    run = prog.launch(grid, [dK, dS, dH], [], ctx, s)
+    assert run.wait()
+    T = run.launch_ms() / 1e3
+    assert np.array_equal(total(), want)
+    preempted = 0
+    for fr in (0.2, 0.5, 0.8):
+        dH.zero_()
+        torch.cuda.synchronize()
+        st, _, _ = flag_run(prog, grid, [dK, dS, dH], [], ctx, fr * T, s, None)
+        torch.cuda.synchronize()
+        preempted += st["warps_preempted"]
+        assert np.array_equal(total(), want), fr
+    assert preempted > 0
