@@ -288,7 +288,10 @@ def summarize(recs):
         "latency_us_median": float(np.median(lat)), "latency_us_p99": float(np.percentile(lat, 99)),
         "latency_us_max": float(lat.max()),
         "resume_us_median": float(np.median(res)), "resume_us_max": float(res.max()),
+        "resume_us_p99": float(np.percentile(res, 99)),
         "host_latency_us_median": float(np.median([r["host_us"] for r in pre])) if pre else 0.0,
+        "host_latency_us_p99": float(np.percentile([r["host_us"] for r in pre], 99)) if pre else 0.0,
+        "host_latency_us_max": float(max(r["host_us"] for r in pre)) if pre else 0.0,
         "signal_to_drained_us_median": (float(np.median([r["signal_us"] for r in pre if r.get("signal_us") is not None]))
                                         if any(r.get("signal_us") is not None for r in pre) else None),
         "preempted_steps": len(pre), "steps": len(recs),

@@ -1,7 +1,8 @@
-"""A small flag preemption through the CTXB_WATCHER path (+ drain notice,
-gathered resume), for compute-sanitizer: C3 at 1024 x 512 and C4a at 2^16
-keys, preempted by the watcher (no memop fallback), resumed, compared with
-the uninterrupted run."""
+"""A small flag preemption on the library's default path (DESIGN.md 8q:
+CTXB_WATCHER + drain notice + the cost model's poll test, gathered resume for
+atomics), for compute-sanitizer: C2 at 256^3, C3 at 2048 x 1024 and C4a at
+2^16 keys, preempted by the watcher (no memop fallback), resumed, compared
+with the uninterrupted run."""
 import os
 import sys
 import time
@@ -15,8 +16,9 @@ import paper_conf_ipps_jiw21_b200 as cb  # noqa: E402
 from workloads import configs  # noqa: E402
 
 
-def run_case(txt, bufs, out_i, extra):
-    prog = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | cb.WATCHER | cb.DRAIN_NOTICE | extra)
+def run_case(txt, bufs, out_i, extra=0, mb=0):
+    prog = cb.Program(txt, poll_policy=cb.POLL_EXPLICIT, flags=cb.ALL | extra, min_blocks_per_sm=mb)
+    assert prog.info["flags"] & (cb.WATCHER | cb.DRAIN_NOTICE) == cb.WATCHER | cb.DRAIN_NOTICE
     grid = prog.persistent_grid()
     ctx = torch.zeros(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
     s = torch.cuda.Stream()
@@ -43,12 +45,16 @@ def run_case(txt, bufs, out_i, extra):
     return npre
 
 
+c2 = configs.c2(256, 256, 256)
+a, b = (torch.from_numpy(c2["buffers"][n].view(np.int32)).cuda() for n in ("A", "B"))
+print("c2 preempted warps:", run_case(c2["ir"], [a, b, torch.zeros(256 * 256, dtype=torch.int32, device="cuda")], 2,
+                                      mb=c2["min_blocks"]))
 c3 = configs.c3(2048, 1024, 64, **configs.BENCH_C3)
 x = torch.from_numpy(c3["buffers"]["X"].view(np.int32)).cuda()
-print("c3 preempted warps:", run_case(c3["ir"], [x, torch.zeros(2048 * 1024, dtype=torch.int32, device="cuda")], 1, 0))
+print("c3 preempted warps:", run_case(c3["ir"], [x, torch.zeros(2048 * 1024, dtype=torch.int32, device="cuda")], 1))
 c4 = configs.c4a(1 << 16, grid=1)
 k = torch.from_numpy(c4["buffers"]["keys"].view(np.int32)).cuda()
 st = torch.from_numpy(c4["buffers"]["starts"].view(np.int32)).cuda()
 print("c4a preempted warps:", run_case(c4["ir"], [k, st, torch.zeros(256 * 2048, dtype=torch.int32, device="cuda")], 2,
-                                       cb.SYNC_POLL))
+                                       ))
 print("ok")
