@@ -410,16 +410,23 @@ int ctxb_launch(ctxb_program* prog, uint32_t grid_blocks, void* const* buffers,
                 const uint32_t* uniforms, void* ctx_buf, uint64_t ctx_buf_bytes, void* stream,
                 const uint32_t* forced_targets, ctxb_run** out);
 
-/* Raise the preemption signal (the launch's unique signal value written to
- * the master flag word by `ctrl_stream`, which must not be the run's stream;
- * with CTXB_ARMED_SIGNAL by the library's own stream; the warps forward it to
- * the flag replicas they poll), and wait until every warp of the run has
+/* Raise the preemption signal and wait until every warp of the run has
  * either saved its context and exited or finished.  Flags are never
  * reset: the next launch waits for a different value.  Fills `stats` if
  * non-NULL.  stats == NULL returns as soon as the launch drained; the headers
  * are read by the next call that needs the run's state (ctxb_wait / query /
  * resume / read_*), so the GPU is free for other work one host round trip
  * earlier.  _STATE if the run is not running. */
+/* Signal paths: by default (CTXB_WATCHER) a host store that the
+ * launch's watcher warp relays to the flag words; ctrl_stream may be NULL (the
+ * watcher alone) or a stream that also issues the stream-memop write as a
+ * fallback.  Otherwise the launch's unique signal value is written to the
+ * master flag word by `ctrl_stream` (which must not be the run's stream, nor
+ * the legacy stream, nor a blocking stream while the run is on the legacy
+ * stream: _INVALID_ARG), or with CTXB_ARMED_SIGNAL by the library's own
+ * stream; polling warps forward it to the flag replicas they poll.  With
+ * CTXB_DRAIN_NOTICE (default with the watcher) the wait ends on the last
+ * warp's store to host memory. */
 int ctxb_preempt(ctxb_run* run, void* ctrl_stream, ctxb_preempt_stats* stats);
 
 /* Raise the preemption signal and return at once (no drain wait): the host
