@@ -61,6 +61,7 @@ struct ctxb_program {
   double t_an = 0, t_cg = 0, t_cc = 0;
   std::mutex mu;
   std::map<CUcontext, Mod> mods;
+  std::map<CUcontext, uint64_t> gather_resident;   // per context: blocks a gathered resume may wait for
   struct Res {
     CUdeviceptr flag = 0, stamps = 0, forced = 0;
     uint32_t n_warps = 0;
@@ -1229,19 +1230,31 @@ int ctxb_resume(ctxb_run* r, void* stream, const uint32_t* forced_targets) {
   r->rb_target = 0;
   if (r->prog->opt.flags & CTXB_GATHER_RESUME) {
     // wait only for warps that can all be resident at once (persistent grid)
-    Driver& d = driver();
-    int b = 0, n = 0;
-    CUdevice dev;
-    CU(d.cuOccupancyMaxActiveBlocksPerMultiprocessor(&b, r->mod.resume, r->prog->prog.block, 0));
-    CU(d.cuCtxGetDevice(&dev));
-    CU(d.cuDeviceGetAttribute(&n, CU_DEVICE_ATTRIBUTE_MULTIPROCESSOR_COUNT, dev));
-    uint64_t resident = (uint64_t)b * (uint64_t)n;
-    if ((r->prog->opt.flags & CTXB_WATCHER) && !watcher_disabled()) {
-      // the watcher warp takes a slot: a block that cannot be resident beside
-      // it would keep the gathered blocks waiting
-      uint32_t g = 0;
-      if (int rc = ctxb_persistent_grid(r->prog, &g)) return rc;
-      resident = std::min<uint64_t>(resident, g);
+    // blocks that can all be resident at once (a static property of the
+    // program on this context: computed once, off the later resumes' path)
+    uint64_t resident = 0;
+    {
+      std::lock_guard<std::mutex> g(r->prog->mu);
+      auto it = r->prog->gather_resident.find(r->ctx);
+      if (it != r->prog->gather_resident.end()) resident = it->second;
+    }
+    if (!resident) {
+      Driver& d = driver();
+      int b = 0, n = 0;
+      CUdevice dev;
+      CU(d.cuOccupancyMaxActiveBlocksPerMultiprocessor(&b, r->mod.resume, r->prog->prog.block, 0));
+      CU(d.cuCtxGetDevice(&dev));
+      CU(d.cuDeviceGetAttribute(&n, CU_DEVICE_ATTRIBUTE_MULTIPROCESSOR_COUNT, dev));
+      resident = (uint64_t)b * (uint64_t)n;
+      if ((r->prog->opt.flags & CTXB_WATCHER) && !watcher_disabled()) {
+        // the watcher warp takes a slot: a block that cannot be resident beside
+        // it would keep the gathered blocks waiting
+        uint32_t g = 0;
+        if (int rc = ctxb_persistent_grid(r->prog, &g)) return rc;
+        resident = std::min<uint64_t>(resident, g);
+      }
+      std::lock_guard<std::mutex> g(r->prog->mu);
+      r->prog->gather_resident[r->ctx] = resident;
     }
     if ((uint64_t)r->grid <= resident) {
       // target = blocks with >= 1 preempted warp (one global arrival per block)
@@ -1253,7 +1266,7 @@ int ctxb_resume(ctxb_run* r, void* stream, const uint32_t* forced_targets) {
         blocks += any;
       }
       r->rb_target = blocks;
-      CU(d.cuMemsetD32Async(r->flag + 128, 0, 32 + r->grid, r->stream));   // arrivals + release words
+      CU(driver().cuMemsetD32Async(r->flag + 128, 0, 32 + r->grid, r->stream));   // arrivals + release words
     }
   }
   r->epoch++;
