@@ -1111,6 +1111,7 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
         recs, done, wall, bad = loop(arr, seconds)
         waits = np.array([r["wait_ms"] for r in recs]) if recs else np.zeros(1)
         lats = np.array([r["lat_us"] for r in recs if r["lat_us"] is not None]) if recs else np.zeros(0)
+        own = np.array([r["wait_ms"] - r["late_ms"] for r in recs]) if recs else np.zeros(0)
         jobs_base = sum(base_done.values()) / base_wall
         jobs_trace = sum(done.values()) / wall
         busy = len(recs) * ls_ms / 1e3 / wall
@@ -1118,6 +1119,13 @@ def bench_c5(cb, seconds, seed, rank, modes=("ctxback", "full_hw", "none")):
             "arrivals": len(recs), "preemptions": int(len(lats)),
             "ls_wait_ms_p50": float(np.median(waits)), "ls_wait_ms_p99": float(np.percentile(waits, 99)),
             "ls_wait_ms_max": float(waits.max()),
+            # the part the preemption mechanism decides: the wait counted from when the
+            # host loop could act on the arrival (an arrival during the previous LS job
+            # queues behind it, host_to_ls, whatever the mechanism)
+            "ls_wait_after_host_ms_p50": float(np.median(own)) if len(own) else None,
+            "ls_wait_after_host_ms_p99": float(np.percentile(own, 99)) if len(own) else None,
+            "ls_wait_after_host_ms_max": float(own.max()) if len(own) else None,
+            "arrivals_queued_behind_ls": int(sum(1 for r in recs if r["late_ms"] > 0.05)),
             "latency_us_p50": float(np.median(lats)) if len(lats) else None,
             "latency_us_p99": float(np.percentile(lats, 99)) if len(lats) else None,
             "latency_us_max": float(lats.max()) if len(lats) else None,
