@@ -126,3 +126,39 @@ def test_speculative_restore_loads_precede_the_header_test():
     # C2's plans hold 68-70 values: nothing is speculated (register budget)
     c2 = cb.Program(configs.c2(256, 256, 64)["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=2)
     assert "_spec(pay" not in c2.source
+
+
+def _loops(cubin, fn):
+    """(instructions, FFMA, IMAD) of every backward-branch range of `fn`'s SASS."""
+    lines = _cuobjdump(cubin, "-sass", "-fun", fn).splitlines()
+    ins = []
+    for ln in lines:
+        m = re.match(r"\s+/\*([0-9a-f]{4,})\*/\s+(.*?);", ln)
+        if m:
+            ins.append((int(m.group(1), 16), m.group(2)))
+    out = []
+    for a, txt in ins:
+        m = re.search(r"BRA\s+(?:`\(.*?\)\s*)?0x([0-9a-f]+)", txt)
+        if m and int(m.group(1), 16) < a:
+            body = [re.sub(r"^@!?U?P\w+\s+", "", x[1]).split()[0] for x in ins if int(m.group(1), 16) <= x[0] <= a]
+            out.append((len(body), sum(o.startswith("FFMA") for o in body), sum(o.startswith("IMAD") for o in body)))
+    return out
+
+
+def test_c2_resumed_warps_run_the_normal_k_loop():
+    """after the current outer iteration, resumed warps run a
+    k-loop as good as the normal kernel's (no irreducible loop, lane offsets
+    recomputed): the resume kernel has a 256-FFMA loop within 16 instructions
+    of the normal kernel's, with as few address IMADs (it had 64 more)."""
+    cb = _cb()
+    prog = cb.Program(configs.c2()["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=2)
+    cub = prog.cubin()
+    run = [x for x in _loops(cub, "ctxb_run") if x[1] == 256]
+    res = [x for x in _loops(cub, "ctxb_resume") if x[1] == 256]
+    best_run = min(run)
+    best_res = min(res)
+    assert best_res[0] <= best_run[0] + 16, (best_run, res)
+    assert best_res[2] <= best_run[2] + 4, (best_run, res)
+    src = prog.source
+    assert "RT_0:" in src and "copy A of BB" in src and "rm_" not in src
+    assert "kernel-invariant registers recomputed" in src

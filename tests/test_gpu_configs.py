@@ -578,3 +578,35 @@ def test_watcher_lifecycle_fuzz(which, path):
         assert npre > 0
     finally:
         faulthandler.cancel_dump_traceback_later()
+
+
+def test_c2_resumed_kernel_runs_at_normal_speed():
+    """C2 preempted at every warp's first poll visit (forced), so
+    the resume kernel does almost all of the work: bit-exact, and it takes no
+    more than 1.25x the uninterrupted kernel (before the resume code re-entered
+    loops through a peeled copy and recomputed the lane offsets: 3x)."""
+    import torch
+    cb = _cb()
+    cfg = configs.c2()
+    prog = cb.Program(cfg["ir"], poll_policy=cb.POLL_EXPLICIT, debug=cb.DEBUG_FORCED, min_blocks_per_sm=2)
+    grid = prog.persistent_grid()
+    nw = grid * 8
+    dA, dB = (torch.from_numpy(cfg["buffers"][n].view(np.int32)).cuda() for n in ("A", "B"))
+    dC = torch.zeros(4096 * 4096, dtype=torch.int32, device="cuda")
+    ctx = torch.empty(prog.context_capacity(grid), dtype=torch.uint8, device="cuda")
+    never = np.full(nw, cb.NEVER, np.uint32)
+    ts = []
+    for _ in range(3):
+        run = prog.launch(grid, [dA, dB, dC], [], ctx, forced=never)
+        assert run.wait()
+        ts.append(run.launch_ms())
+    ref = dC.clone()
+    dC.zero_()
+    run = prog.launch(grid, [dA, dB, dC], [], ctx, forced=np.full(nw, 1, np.uint32))
+    assert not run.wait()
+    run.resume(forced=never)
+    assert run.wait()
+    t_res = run.launch_ms()
+    torch.cuda.synchronize()
+    assert torch.equal(dC, ref)
+    assert t_res < 1.25 * float(np.median(ts)), (t_res, ts)
