@@ -80,6 +80,25 @@ def test_analyzer_parity_random(seed):
     _same_plans(txt)
 
 
+@pytest.mark.parametrize("seed", range(12))
+def test_analyzer_parity_random_loop_nests(seed):
+    txt, _ = random_program(700 + seed, loop=True, nested=True, n_body=8)
+    _same_plans(txt)
+
+
+def test_resume_code_of_a_loop_nest():
+    """a site inside the inner loop of a nest resumes through
+    RT_k and a peeled copy of the whole nest, whose branches to the nest's
+    header go back to the normal code."""
+    txt, _ = random_program(5, loop=True, nested=True, n_body=6)
+    p = cb.Program(txt, debug=cb.DEBUG_FORCED | cb.DEBUG_NO_COMPILE)
+    src = p.source
+    assert "RT_" in src and "copy A of BB1..BB4" in src
+    copy_a = src[src.index("copy A of BB1..BB4"):]
+    copy_a = copy_a[:copy_a.index("\n}\n")]
+    assert "goto BA2;" in copy_a and "goto BB1;" in copy_a and "goto BA1;" not in copy_a
+
+
 @pytest.mark.parametrize("flags", [0, 1, 3, 5, 7])
 def test_analyzer_parity_technique_toggles(flags):
     for seed in range(8):

@@ -101,6 +101,21 @@ def test_random_programs(seed):
     check(txt, grid, bufs, scheds)
 
 
+@pytest.mark.parametrize("seed", range(6))
+def test_random_loop_nests(seed):
+    """Loop nests: resumes inside the inner and the outer loop
+    go through RT_k and the peeled copy of the nest; forced, nested, poisoned."""
+    txt, size = random_program(700 + seed, loop=True, nested=True, n_body=8)
+    op = ir.parse(txt)
+    grid = 2
+    nout = op.nv - 1 + op.ns - 2
+    bufs = random_buffers(seed, op.block, grid, size, nout)
+    r = np.random.default_rng(seed)
+    nw = grid * op.nwarps
+    scheds = [[r.integers(0, 90, nw).astype(np.uint32), r.integers(0, 40, nw).astype(np.uint32)] for _ in range(6)]
+    check(txt, grid, bufs, scheds)
+
+
 @pytest.mark.parametrize("name", ["fig2", "fig3", "fig4", "fig5", "fig6", "r9", "r3", "r3bar", "osrb_select", "n3"])
 def test_paper_figures_on_gpu(name):
     import json

@@ -29,15 +29,16 @@ def main(first, n, seconds):
     for seed in range(first, first + n):
         if time.time() > t_end:
             break
-        loop = seed % 3 == 0
-        txt, size = random_program(seed, loop=loop, n_body=10 + seed % 7)
+        loop = seed % 3 == 0 or seed % 5 == 0
+        nested = loop and seed % 2 == 0          # loop nests
+        txt, size = random_program(seed, loop=loop, nested=nested, n_body=10 + seed % 7)
         op = ir.parse(txt)
         grid = 1 + seed % 3
-        nout = op.nv - 1 + op.ns - (1 if loop else 0)
+        nout = op.nv - 1 + op.ns - (1 if loop else 0) - (1 if nested else 0)
         bufs = random_buffers(seed, op.block, grid, size, nout)
         r = np.random.default_rng(seed)
         nw = grid * op.nwarps
-        scheds = [[r.integers(0, 60, nw).astype(np.uint32), r.integers(0, 20, nw).astype(np.uint32)]
+        scheds = [[r.integers(0, 90, nw).astype(np.uint32), r.integers(0, 30, nw).astype(np.uint32)]
                   for _ in range(3)]
         name, flags, mode = VARIANTS[seed % len(VARIANTS)]
         try:

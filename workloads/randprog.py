@@ -172,15 +172,19 @@ class _Gen:
 
 def random_program(seed: int, nv: int = 6, ns: int = 2, n_body: int = 12, loop: bool = False,
                    block: int = 64, mem_ops: bool = True, fp: bool = True, atomics: bool = False,
-                   nblocks_hint: int = 2):
+                   nblocks_hint: int = 2, nested: bool = False):
     """Return IR text.  Buffers: ro0, ro1 (size = block*nblocks_hint), rw0
-    (same size), scr (wo scratch), out (wo, (nv+ns) words per thread)."""
+    (same size), scr (wo scratch), out (wo, (nv+ns) words per thread).
+    loop: the first body block is a counted loop; nested (with loop): an
+    outer counted loop (2 trips) around all body blocks, its header holding
+    the inner loop's counter set-up (a loop nest, as in C2's tile / k loops)."""
     g = _Gen(seed, nv, ns, n_body, loop, block, mem_ops, fp, atomics)
     size = 1
     while size < block * nblocks_hint:
         size *= 2
     hdr = [".kernel rnd%d" % seed, ".buffer ro ro0", ".buffer ro ro1", ".buffer rw rw0",
-           ".buffer wo scr", ".buffer wo out", f".vregs {nv}", f".sregs {ns + (1 if loop else 0)}",
+           ".buffer wo scr", ".buffer wo out", f".vregs {nv}",
+           f".sregs {ns + (1 if loop else 0) + (1 if loop and nested else 0)}",
            f".block {block}"]
     g.lines.append("init:")
     for i in range(nv):
@@ -190,6 +194,10 @@ def random_program(seed: int, nv: int = 6, ns: int = 2, n_body: int = 12, loop: 
         g.emit(f"ldg s{i}, ro{i % 2}[s{i}]")
     ctr = f"s{ns}"
     nblk = 1 + int(g.r.integers(3))
+    outer = f"s{ns + 1}" if (loop and nested) else None
+    if outer:
+        g.emit(f"mov {outer}, 2")
+        g.lines.append("outer:")
     for b in range(nblk):
         is_loop = loop and b == 0
         if is_loop:
@@ -206,6 +214,9 @@ def random_program(seed: int, nv: int = 6, ns: int = 2, n_body: int = 12, loop: 
         if is_loop:
             g.emit(f"isub {ctr}, {ctr}, 1")
             g.emit(f"brnz {ctr}, b{b}")
+    if outer:
+        g.emit(f"isub {outer}, {outer}, 1")
+        g.emit(f"brnz {outer}, outer")
     g.lines.append("fin:")
     nout = nv + ns
     # store every register: out[tid * nout + k]; use a fresh index register
