@@ -82,7 +82,7 @@ def test_analyzer_parity_random(seed):
 
 @pytest.mark.parametrize("seed", range(12))
 def test_analyzer_parity_random_loop_nests(seed):
-    txt, _ = random_program(700 + seed, loop=True, nested=True, n_body=8)
+    txt, _ = random_program(700 + seed, loop=True, nested=True, n_body=8, indexed=seed % 3)
     _same_plans(txt)
 
 

@@ -116,6 +116,21 @@ def test_random_loop_nests(seed):
     check(txt, grid, bufs, scheds)
 
 
+@pytest.mark.parametrize("seed,indexed", [(s, 1 + s % 2) for s in range(6)])
+def test_random_indexed_loops(seed, indexed):
+    """Loop-carried index bases: resumed iterations run the fast
+    path (bases < 2^31, masked) or, with a top-bit-set base whose `+ c` wraps
+    into range, the generic path; forced, nested, poisoned; bit-exact."""
+    txt, size = random_program(800 + seed, loop=True, nested=seed % 3 == 0, indexed=indexed, n_body=10)
+    op = ir.parse(txt)
+    grid = 2
+    bufs = random_buffers(seed, op.block, grid, size, txt.count("stg out["))
+    r = np.random.default_rng(seed)
+    nw = grid * op.nwarps
+    scheds = [[r.integers(0, 90, nw).astype(np.uint32), r.integers(0, 40, nw).astype(np.uint32)] for _ in range(6)]
+    check(txt, grid, bufs, scheds)
+
+
 @pytest.mark.parametrize("name", ["fig2", "fig3", "fig4", "fig5", "fig6", "r9", "r3", "r3bar", "osrb_select", "n3"])
 def test_paper_figures_on_gpu(name):
     import json

@@ -31,10 +31,11 @@ def main(first, n, seconds):
             break
         loop = seed % 3 == 0 or seed % 5 == 0
         nested = loop and seed % 2 == 0          # loop nests
-        txt, size = random_program(seed, loop=loop, nested=nested, n_body=10 + seed % 7)
+        indexed = (seed // 2) % 3 if loop else 0  # loop-carried index bases (8r fast / generic path)
+        txt, size = random_program(seed, loop=loop, nested=nested, indexed=indexed, n_body=10 + seed % 7)
         op = ir.parse(txt)
         grid = 1 + seed % 3
-        nout = op.nv - 1 + op.ns - (1 if loop else 0) - (1 if nested else 0)
+        nout = txt.count("stg out[")
         bufs = random_buffers(seed, op.block, grid, size, nout)
         r = np.random.default_rng(seed)
         nw = grid * op.nwarps

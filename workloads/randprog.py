@@ -172,16 +172,23 @@ class _Gen:
 
 def random_program(seed: int, nv: int = 6, ns: int = 2, n_body: int = 12, loop: bool = False,
                    block: int = 64, mem_ops: bool = True, fp: bool = True, atomics: bool = False,
-                   nblocks_hint: int = 2, nested: bool = False):
+                   nblocks_hint: int = 2, nested: bool = False, indexed: int = 0):
     """Return IR text.  Buffers: ro0, ro1 (size = block*nblocks_hint), rw0
     (same size), scr (wo scratch), out (wo, (nv+ns) words per thread).
     loop: the first body block is a counted loop; nested (with loop): an
     outer counted loop (2 trips) around all body blocks, its header holding
-    the inner loop's counter set-up (a loop nest, as in C2's tile / k loops)."""
+    the inner loop's counter set-up (a loop nest, as in C2's tile / k loops).
+    indexed (with loop): the loop body also loads through `iadd t, base, c`
+    from loop-carried index registers advanced at the end of the body (C2's
+    A / B index pattern); 1: a base in [0, size/2); 2: also a
+    base with its top bit set whose `+ c` wraps (mod 2^32) into range."""
     g = _Gen(seed, nv, ns, n_body, loop, block, mem_ops, fp, atomics)
     size = 1
     while size < block * nblocks_hint:
         size *= 2
+    ix = loop and indexed > 0
+    vA, vW = f"v{nv + 1}", f"v{nv + 2}"
+    half = max(1, size // 2)
     hdr = [".kernel rnd%d" % seed, ".buffer ro ro0", ".buffer ro ro1", ".buffer rw rw0",
            ".buffer wo scr", ".buffer wo out", f".vregs {nv}",
            f".sregs {ns + (1 if loop else 0) + (1 if loop and nested else 0)}",
@@ -192,6 +199,10 @@ def random_program(seed: int, nv: int = 6, ns: int = 2, n_body: int = 12, loop: 
     for i in range(ns):
         g.emit(f"and s{i}, %ctaid, {size - 1}")
         g.emit(f"ldg s{i}, ro{i % 2}[s{i}]")
+    if ix:
+        g.emit(f"and {vA}, %tid, {half - 1}")
+        if indexed > 1:
+            g.emit(f"iadd {vW}, %laneid, 0xFFFFFFC0")
     ctr = f"s{ns}"
     nblk = 1 + int(g.r.integers(3))
     outer = f"s{ns + 1}" if (loop and nested) else None
@@ -205,12 +216,26 @@ def random_program(seed: int, nv: int = 6, ns: int = 2, n_body: int = 12, loop: 
         g.lines.append(f"b{b}:")
         for _ in range(n_body):
             k = int(g.r.integers(10))
+            if is_loop and ix and k < 3:
+                t, d = g.vreg(), g.vreg()
+                if indexed > 1 and k == 0:
+                    g.emit(f"iadd {t}, {vW}, {64 + int(g.r.integers(0, 64))}")
+                    g.emit(f"ldg {d}, ro1[{t}]")
+                else:
+                    g.emit(f"iadd {t}, {vA}, {int(g.r.integers(0, half))}")
+                    g.emit(f"ldg {d}, ro0[{t}]")
+                g.fmag.pop(t, None)
+                g.dst(d)
+                continue
             if mem_ops and k < 2:
                 g.memop(2, size)
             elif fp and k < 4:
                 g.fpop()
             else:
                 g.alu(scalar=(ns > 0 and k == 9))
+        if is_loop and ix:
+            g.emit(f"iadd {vA}, {vA}, 1")
+            g.emit(f"and {vA}, {vA}, {half - 1}")
         if is_loop:
             g.emit(f"isub {ctr}, {ctr}, 1")
             g.emit(f"brnz {ctr}, b{b}")
@@ -221,7 +246,7 @@ def random_program(seed: int, nv: int = 6, ns: int = 2, n_body: int = 12, loop: 
     nout = nv + ns
     # store every register: out[tid * nout + k]; use a fresh index register
     # computed from %tid so no program register is disturbed before its store
-    hdr[6] = f".vregs {nv + 1}"
+    hdr[6] = f".vregs {nv + 1 + (2 if ix else 0)}"
     t = f"v{nv}"
     g.emit(f"imad {t}, %ctaid, %ntid, %tid")
     g.emit(f"imul {t}, {t}, {nout}")
