@@ -25,6 +25,11 @@ def setups():
     yield "c2", c2["ir"], 2, [A, B, C]
     if os.environ.get("ONLY_C2"):
         return
+    c2s = configs.c2s()
+    A2, B2 = (torch.from_numpy(c2s["buffers"][n].view(np.int32)).cuda() for n in ("A", "B"))
+    yield "c2s", c2s["ir"], c2s.get("min_blocks", 0), [A2, B2, torch.zeros(4096 * 4096, dtype=torch.int32, device="cuda")]
+    if os.environ.get("ONLY_C2S"):
+        return
     c3 = configs.c3(**configs.BENCH_C3)
     X = torch.from_numpy(c3["buffers"]["X"].view(np.int32)).cuda()
     yield "c3", c3["ir"], 0, [X, torch.zeros(c3["W"] * c3["H"], dtype=torch.int32, device="cuda")]
