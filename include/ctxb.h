@@ -105,7 +105,9 @@ extern "C" {
                              value loaded flag_depth sites earlier: detection
                              within one site interval instead of flag_depth + 1,
                              for loops whose iterations are long (C4a)         */
-#define CTXB_HOST_SIGNAL 512u /* runtime + codegen: ctxb_preempt also raises a word
+#define CTXB_HOST_SIGNAL 512u /* (A/B study option, superseded by the default
+                             CTXB_WATCHER path of DESIGN.md 8q.)
+                             runtime + codegen: ctxb_preempt also raises a word
                              in mapped pinned host memory.  Each warp reads it
                              (system-scope load over PCIe, tested one site
                              later) once every ceil(n_warps / R) of its polls,
@@ -119,7 +121,9 @@ extern "C" {
                              mode only (ignored by CTXB_DEBUG_FORCED).
                              stats.signal_to_drained_us is 0 in this mode (the
                              host store is not stream-ordered): use host_us   */
-#define CTXB_ARMED_SIGNAL 1024u /* runtime: every launch (and resume) pre-enqueues
+#define CTXB_ARMED_SIGNAL 1024u /* (A/B option, superseded by the default CTXB_WATCHER
+                             path of DESIGN.md 8q: -12 µs host latency on C2.)
+                             runtime: every launch (and resume) pre-enqueues
                              its preemption signal on a library-owned
                              greatest-priority stream: cuStreamWaitValue32 on a
                              gate word in mapped pinned host memory, then the
@@ -138,7 +142,9 @@ extern "C" {
                              stores the warp-uniform value, the preemption
                              routine reads it after __syncwarp().  Plans and
                              bytes unchanged                                  */
-#define CTXB_OSRB_LANES 4096u /* codegen: OSRB backup j lives in lane j % 32 of one
+#define CTXB_OSRB_LANES 4096u /* (A/B option: slower than the default register slot,
+                             DESIGN.md 8k.)
+                             codegen: OSRB backup j lives in lane j % 32 of one
                              register per 32 backups (the paper's VGPR-lane
                              tier), read back with a warp shuffle in the
                              (converged) preemption routine.  Exclusive with
