@@ -583,7 +583,7 @@ def test_watcher_lifecycle_fuzz(which, path):
 def test_c2_resumed_kernel_runs_at_normal_speed():
     """C2 preempted at every warp's first poll visit (forced), so
     the resume kernel does almost all of the work: bit-exact, and it takes no
-    more than 1.25x the uninterrupted kernel (before the resume code re-entered
+    more than 1.10x the uninterrupted kernel (measured 1.01x; before the resume code re-entered
     loops through a peeled copy and recomputed the lane offsets: 3x)."""
     import torch
     cb = _cb()
@@ -609,4 +609,4 @@ def test_c2_resumed_kernel_runs_at_normal_speed():
     t_res = run.launch_ms()
     torch.cuda.synchronize()
     assert torch.equal(dC, ref)
-    assert t_res < 1.25 * float(np.median(ts)), (t_res, ts)
+    assert t_res < 1.10 * float(np.median(ts)), (t_res, ts)
